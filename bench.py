@@ -1,0 +1,372 @@
+#!/usr/bin/env python
+"""bench.py -- the unified graph operator on B200 (one JSON line on rank 0).
+
+Default workload (BASELINE.json configs[4], the largest single-GPU config and the one the
+north-star target is quoted on): C5 Reddit-shaped synthetic graph (232,965 v / 114,615,892 e),
+copy_u_sum at F = 602 (GraphSage/GCN-style aggregation, Fig. 4).
+
+A "step" is one full call of the operator (ug_op_run: every kernel it enqueues) over the
+whole graph with inputs resident in HBM; N > 1 (torchrun) shards destination rows by edge
+count, and a step is the NCCL all-gather of X plus the local op.
+
+  value         effective GB/s = logical algorithmic bytes / device time
+  e2e           same metric through the public API with host (pinned) X in and Y out
+  roofline      the dominant kernel (main traversal) timed with CUDA events inside the
+                timed region, algorithmic bytes / its average duration vs measured HBM peak
+  cpu_baseline  the CPU oracle (oracle/, 1 core) on a bounded row sample, same metric
+  --impl reference   times the oracle alone (this tier's reference arm)
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "graph-op latency and effective HBM GB/s vs ~8 TB/s, per op×graph, 1/2/4/8 GPU"
+OPS = {  # name -> (edge_op, gather_op, A type, B type)
+    "copy_u_sum": ("copy_lhs", "sum", "u", None),
+    "copy_u_mean": ("copy_lhs", "mean", "u", None),
+    "copy_u_max": ("copy_lhs", "max", "u", None),
+    "u_mul_e_sum": ("mul", "sum", "u", "e"),
+    "u_dot_v": ("dot", "assign", "u", "v"),
+}
+
+
+def logical_bytes(V, E, F, op, H=1):
+    """4(V+1) row_ptr + 4E col_idx + 4 E w per u/e operand + 4 V w per v operand
+    + output (4 V F for C = v, 4 E w_out for C = e)."""
+    eo, go, a, b = OPS[op]
+    B = 4 * (V + 1) + 4 * E
+    for t, w in ((a, F), (b, 1 if op == "u_mul_e_sum" else F)):
+        if t in ("u", "e"):
+            B += 4 * E * w
+        elif t == "v":
+            B += 4 * V * w
+    B += 4 * E * H if go == "assign" else 4 * V * F
+    return B
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) == 6:
+                self.rows.append(parts)
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[2 + i] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+# ---------------------------------------------------------------------------- CPU oracle
+def oracle_sample(cfg_name, op, F, src, dst, V, target_s=15.0, seed=0):
+    """Time the oracle (1 core) on a bounded random sample of destination rows; returns
+    (GB/s in the same logical-byte metric, rows, edges, seconds)."""
+    import oracle
+    import ugdata
+    eo, go, a, b = OPS[op]
+    rng = np.random.default_rng(seed)
+    deg = np.bincount(dst, minlength=V)
+    mean_deg = max(1.0, float(deg.mean()))
+    # calibrate: ~2 ns per (edge x feature) element for the plain oracle, then measure
+    n_rows = int(max(16, min(V, target_s / (8e-9 * mean_deg * F))))
+    rows = np.sort(rng.choice(V, size=n_rows, replace=False)).astype(np.int64)
+    sub = np.nonzero(np.isin(dst, rows))[0]
+    X = ugdata.values(V, F, 99, 1)
+    w = ugdata.values(len(sub), 1, 99, 2, role="edge") if b == "e" else None
+    s_src, s_dst = src[sub], dst[sub]
+    t0 = time.perf_counter()
+    if go == "assign":
+        oracle.op(V, s_src, s_dst, eo, go, A=X, a_type=a, B=X, b_type=b, c_type="e", F=F, H=1)
+        Es, Vs = len(sub), 0
+    else:
+        oracle.op(V, s_src, s_dst, eo, go, A=X, a_type=a, B=w, b_type=b, c_type="v", F=F, H=1, rows=rows)
+        Es, Vs = len(sub), len(rows)
+    dt = time.perf_counter() - t0
+    by = logical_bytes(Vs, Es, F, op)
+    return by / dt / 1e9, len(rows), Es, dt
+
+
+def cores_used():
+    return 1
+
+
+# ---------------------------------------------------------------------------- GPU run
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C5")
+    ap.add_argument("--op", default="copy_u_sum", choices=sorted(OPS))
+    ap.add_argument("--F", type=int, default=None)
+    ap.add_argument("--schedule", default=None, help="Table 9 notation; default: ug_schedule_select")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    world, rank, local = dist_env()
+    import ugdata
+    cfg = ugdata.CONFIGS[args.config]
+    F = args.F or cfg.widths[-1]
+    workload = f"{args.config} {cfg.label} synthetic graph ({cfg.V:,} v / {cfg.E:,} e), {args.op}, F={F}"
+
+    if args.impl == "reference":
+        run_reference(args, cfg, F, workload, world, rank)
+        return
+
+    import torch
+    import paper_conf_asplos_0001lslwlgslllw23_b200 as ug
+
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local if world > 1 else 0)
+    torch.cuda.set_device(dev)
+
+    src, dst = ugdata.graph(args.config)
+    V, E = cfg.V, len(src)
+    eo, go, a_t, b_t = OPS[args.op]
+    g_full = ug.Graph(V, src, dst)
+
+    # shard: edge-balanced destination rows (R21); X row blocks of ceil(V/P) for the all-gather
+    if world > 1:
+        splits = g_full.partition(world)
+        r0, r1 = int(splits[rank]), int(splits[rank + 1])
+        g = g_full.view_rows(r0, r1)
+    else:
+        r0, r1 = 0, V
+        g = g_full
+    Vl = r1 - r0
+    blk = -(-V // world)
+    X_host = ugdata.values(V, F, cfg.seed + 1, 1)
+    X_full = torch.empty(blk * world, F, device=dev)
+    X_full[:V].copy_(torch.from_numpy(X_host))
+    X_local = X_full[rank * blk:(rank + 1) * blk].clone() if world > 1 else None
+    Bt = None
+    if b_t == "e":
+        rp = g_full.csr()[0] if world > 1 else None
+        wE = torch.from_numpy(ugdata.values(E, 1, cfg.seed + 1, 2, role="edge")).to(dev)
+        Bt = wE[int(rp[r0]):int(rp[r1])] if world > 1 else wE
+    elif b_t == "v":
+        Bt = X_full[r0:r1]
+    Y = torch.empty(Vl if go != "assign" else g.stats()["E"], F if eo != "dot" else 1, device=dev)
+    sched = args.schedule
+    kw = dict(A=X_full[:V], a_type=a_t, B=Bt, b_type=b_t, C=Y, c_type="e" if go == "assign" else "v",
+              F=F, H=1)
+    chosen = sched or ug.schedule_select(g, eo, go, **kw)
+    launches = ug.launch_count(g, eo, go, schedule=chosen, **kw)
+
+    stream = torch.cuda.current_stream(dev)
+    ev_k0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ev_k1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ev_s0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ev_s1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    for e in ev_k0 + ev_k1:
+        e.record(stream)   # materialise the cudaEvent_t handles
+    torch.cuda.synchronize()
+
+    def step(i=None):
+        if world > 1:
+            dist.all_gather_into_tensor(X_full, X_local)
+        if i is None:
+            ug.op_run(g, eo, go, schedule=chosen, **kw)
+        else:
+            ug.op_run_events(g, eo, go, ev_k0[i], ev_k1[i], schedule=chosen, **kw)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clocks:
+        for i in range(args.steps):
+            ev_s0[i].record(stream)
+            step(i)
+            ev_s1[i].record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    step_ms = [ev_s0[i].elapsed_time(ev_s1[i]) for i in range(args.steps)]
+    kern_ms = [ev_k0[i].elapsed_time(ev_k1[i]) for i in range(args.steps)]
+    tot = sum(step_ms)
+    ktot = sum(kern_ms)
+    if world > 1:
+        t = torch.tensor([tot, ktot], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        tot, ktot = float(t[0]), float(t[1])
+    ms = tot / args.steps
+    kms = ktot / args.steps
+    by = logical_bytes(V, E, F, args.op)
+    by_local = logical_bytes(Vl, g.stats()["E"], F, args.op)
+    value = by / (ms * 1e-3) / 1e9
+    peak, peak_src = load_peaks()
+    achieved = by_local / (kms * 1e-3) / 1e9
+
+    # e2e through the public API: pinned host X -> device, op, device Y -> pinned host.
+    e2e = None
+    if not args.no_e2e and world == 1:
+        Xh = torch.from_numpy(X_host).pin_memory()
+        Yh = torch.empty(Y.shape, dtype=torch.float32).pin_memory()
+        Xd = torch.empty(V, F, device=dev)
+        kwe = dict(kw)
+        kwe["A"] = Xd
+        if b_t == "v":
+            kwe["B"] = Xd
+        for _ in range(2):
+            Xd.copy_(Xh, non_blocking=True)
+            ug.op_run(g, eo, go, schedule=chosen, **kwe)
+            Yh.copy_(Y, non_blocking=True)
+        torch.cuda.synchronize()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        n_e2e = max(3, min(args.steps, 5))
+        e0.record(stream)
+        for _ in range(n_e2e):
+            Xd.copy_(Xh, non_blocking=True)
+            ug.op_run(g, eo, go, schedule=chosen, **kwe)
+            Yh.copy_(Y, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        e_ms = e0.elapsed_time(e1) / n_e2e
+        e2e = {"value": round(by / (e_ms * 1e-3) / 1e9, 1), "unit": "GB/s", "ms_per_step": round(e_ms, 3),
+               "h2d_bytes_per_step": int(Xh.numel() * 4), "d2h_bytes_per_step": int(Yh.numel() * 4)}
+
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        try:
+            tj = json.load(open(tp))
+            key = f"{args.config}:{args.op}:{F}:{chosen}"
+            traffic = tj.get(key)
+        except (ValueError, OSError):
+            traffic = None
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        gbs, nr, ne, dt = oracle_sample(args.config, args.op, F, src, dst, V)
+        cpu = {"value": round(gbs, 4), "unit": "GB/s", "cores": cores_used(), "kind": "oracle",
+               "sample": f"{args.op} on {nr} random dst rows ({ne} in-edges) of {args.config}, {dt:.1f} s, "
+                         f"oracle/ug_oracle.c single thread"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 1), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": workload, "op": args.op, "V": V, "E": E, "F": F, "ld": F,
+                       "schedule": chosen, "graph": "Chung-Lu lognormal degrees (ugdata), seed %d" % cfg.seed,
+                       "l2": "inputs larger than L2 (X %.0f MB, col_idx %.0f MB > 126 MB): no flush"
+                             % (V * F * 4 / 1e6, E * 4 / 1e6),
+                       "parallelism": f"dst-row sharding x{world}" + (" + NCCL all-gather of X" if world > 1 else ""),
+                       "logical_bytes": by},
+            "latency_ms": round(ms, 4),
+            "frac_of_8TBps": round(value / 8000.0, 4),
+            "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                         "frac": round(achieved / peak, 4), "traffic": traffic,
+                         "kernel": "k_split (SV main traversal)" if chosen.startswith("SV") else "main traversal",
+                         "kernel_ms": round(kms, 4), "peak_source": peak_src,
+                         "bytes": "algorithmic (SURVEY 8(d)) per launch"},
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches * args.steps,
+            "clocks": clocks.summary(),
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def run_reference(args, cfg, F, workload, world, rank):
+    """This tier's reference arm: the CPU oracle as it stands, 1 core, bounded row samples."""
+    if rank != 0:
+        return
+    import ugdata
+    src, dst = ugdata.graph(args.config)
+    V = cfg.V
+    per_step = 60.0 / max(1, args.steps + args.warmup)
+    for i in range(args.warmup):
+        oracle_sample(args.config, args.op, F, src, dst, V, target_s=min(per_step, 5.0), seed=100 + i)
+    vals, rows, edges, secs = [], 0, 0, 0.0
+    for i in range(args.steps):
+        gbs, nr, ne, dt = oracle_sample(args.config, args.op, F, src, dst, V, target_s=min(per_step, 10.0), seed=i)
+        vals.append(gbs)
+        rows += nr
+        edges += ne
+        secs += dt
+    value = float(np.mean(vals))
+    sample = f"{args.op} on {args.steps} random samples ({rows} dst rows, {edges} in-edges total) of {args.config}"
+    line = {"metric": METRIC, "value": round(value, 4), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(secs / args.steps * 1e3, 2), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic", "impl": "reference",
+            "config": {"workload": workload, "op": args.op, "V": V, "E": cfg.E, "F": F},
+            "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,216 @@
+/*
+ * ug.h -- C ABI of libugraph: the unified GNN graph operator of uGrapher
+ * (Zhou et al., ASPLOS'23; text at PAPER.md) re-designed for B200 (sm_100a).
+ *
+ * One call computes, for every destination vertex dst, every in-edge e = (src -> dst) and
+ * every feature f (Fig. 5, lines 14-19):
+ *     tmp = edge_op(A[a_idx][f], B[b_idx][f]);   C[c_idx][f] = gather_op(C[c_idx][f], tmp)
+ * where a_idx/b_idx/c_idx follow the operand's tensor type (type_idx_dict):
+ * Src_V -> src, Dst_V -> dst, Edge -> edge id.  The op set is Table 4
+ * plus `dot` (R5): all 160 DGL graph operators of Table 2.
+ *
+ * Conventions (all entry points):
+ *   - No exceptions cross this boundary; every function returns a ug_status.
+ *   - Feature tensors are fp32, row-major, row stride `ld` (elements, ld >= width).
+ *     Vertex ids and CSR arrays are int32.  Edge id = position in the COO given to
+ *     ug_graph_create (R9).  E < 2^31.
+ *   - Pointers marked "device" must be CUDA device (or managed) memory of the current
+ *     device; "host" pointers are plain host memory.  `stream` is a cudaStream_t (NULL =
+ *     legacy default stream).
+ *   - The library never keeps a caller pointer after a call returns (graphs copy their
+ *     input).  The caller owns A, B, C.
+ *   - ug_op_run is asynchronous (no host synchronisation) and re-entrant across streams;
+ *     graphs are immutable after creation.
+ */
+#ifndef UG_H_
+#define UG_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    UG_OK = 0,
+    UG_ERR_INVALID_ARG = 1,         /* NULL pointer, negative size, bad enum value        */
+    UG_ERR_UNSUPPORTED_OP = 2,      /* op/type combination outside the supported op set  */
+    UG_ERR_SHAPE = 3,               /* operand width not F or H, H does not divide F, ...   */
+    UG_ERR_INDEX_RANGE = 4,         /* vertex id outside [0, V) at graph creation           */
+    UG_ERR_ALIGNMENT = 5,           /* forced vector width incompatible with ld / pointer   */
+    UG_ERR_OOM = 6,                 /* allocation failed                                    */
+    UG_ERR_CUDA = 7,                /* a CUDA call failed; see ug_last_error()              */
+    UG_ERR_UNSUPPORTED_SCHEDULE = 8 /* schedule parameters outside the implemented space    */
+} ug_status;
+
+/* edge_op list of Fig. 5 ("copy_lns/rns" read as copy_lhs/copy_rhs) + dot (R5). */
+typedef enum {
+    UG_EDGE_COPY_LHS = 0, UG_EDGE_COPY_RHS = 1, UG_EDGE_ADD = 2, UG_EDGE_SUB = 3,
+    UG_EDGE_MUL = 4, UG_EDGE_DIV = 5, UG_EDGE_DOT = 6
+} ug_edge_op;
+
+/* gather_op list of Fig. 5.  The paper's copy_rhs used as a gather is an
+ * assignment onto edges (message creation, Table 4 rows 1-5; reading R3). */
+typedef enum {
+    UG_GATHER_ASSIGN = 0, UG_GATHER_SUM = 1, UG_GATHER_MAX = 2, UG_GATHER_MIN = 3,
+    UG_GATHER_MEAN = 4
+} ug_gather_op;
+
+/* tensor_type_list / type_idx_dict. */
+typedef enum { UG_T_NULL = 0, UG_T_SRC_V = 1, UG_T_DST_V = 2, UG_T_EDGE = 3 } ug_ttype;
+
+/* One operand.  data: device fp32; rows implied by type (V for Src_V/Dst_V, E for Edge);
+ * width in {F, H} (H: per-head value broadcast over the head's D = F/H features, R6);
+ * ld >= width, in elements.  The output C of a dot op has width H. */
+typedef struct {
+    void *data;
+    int32_t type;   /* ug_ttype */
+    int32_t width;
+    int64_t ld;
+} ug_tensor;
+
+/* op_info of PAPER.md:385-386: [edge_op, gather_op, A, A_Type, B, B_Type, C, C_Type]
+ * plus the feature width F and head count H (H | F; H = 1 for scalar broadcasts). */
+typedef struct {
+    int32_t edge_op;    /* ug_edge_op   */
+    int32_t gather_op;  /* ug_gather_op */
+    ug_tensor A, B, C;
+    int32_t feat;       /* F */
+    int32_t heads;      /* H */
+} ug_op_info;
+
+/* parallel_strategy of PAPER.md:387-388 and Fig. 6; BV/BE are block-level extensions
+ * (north star).  Notation of Table 9: TE_G1_T16 = {UG_TE, 1, 16}. */
+typedef enum {
+    UG_SCHED_AUTO = 0,
+    UG_TV = 1,      /* thread-vertex: T threads share one dst row's features, owner computes   */
+    UG_TE = 2,      /* thread-edge:   T threads share one edge's features, atomics into dst    */
+    UG_WV = 3,      /* warp-vertex:   T warps per dst row                                       */
+    UG_WE = 4,      /* warp-edge:     T warps per edge                                          */
+    UG_BV = 5,      /* block-vertex:  one CTA per G rows, its warps split each row's edges     */
+    UG_BE = 6,      /* block-edge:    one CTA per G x warps edges, contiguous, segmented reduce */
+    UG_SV = 7       /* split-vertex (B200): rows cut into <= `group` edge chunks, column tiles of
+                       `ftile` features in tile-major order (L2-resident), partials fixed up   */
+} ug_strategy;
+
+typedef struct {
+    int32_t strategy;       /* ug_strategy                                                      */
+    int32_t group;          /* G: units per thread/warp group (V/E grouping);
+                               UG_SV: max edges per row chunk                                    */
+    int32_t tile;           /* T: feature tiling: threads (TV/TE) or warps (WV/WE)
+                               sharing one unit's features                                       */
+    int32_t block_threads;  /* CTA size (0 -> 256)                                              */
+    int32_t ftile;          /* column-tile width for L2 blocking, tile-major grid order; 0 = off */
+    int32_t vec;            /* feature vector width 1/2/4; 0 -> widest the layout allows        */
+} ug_schedule;
+
+/* Optional allocator for graph-owned device arrays (e.g. torch's caching allocator).
+ * NULL -> cudaMallocAsync / cudaFreeAsync on the given stream. */
+typedef struct {
+    void *(*alloc)(size_t bytes, void *ctx, void *stream);
+    void (*free)(void *ptr, void *ctx, void *stream);
+    void *ctx;
+} ug_allocator;
+
+typedef struct ug_graph ug_graph;
+
+/* Graph creation flags. */
+#define UG_GRAPH_HOST_ONLY 1   /* build and keep the CSR on the host only (no CUDA calls):
+                                  for host-side partitioning, stats, selection and tests  */
+
+/*
+ * ug_graph_create -- COO -> in-CSR keyed by destination (get_inedges).
+ *   num_vertices V >= 0, num_edges E in [0, 2^31); src[E], dst[E] int32 vertex ids.
+ *   on_device: 1 if src/dst are device pointers, 0 if host.
+ *   Builds row_ptr[V+1], col_idx[E] = src sorted stably by dst (edge-id order inside a
+ *   row, R10), eid[E] (omitted when the COO is already dst-sorted), dst_of[E] (COO row array
+ *   for edge-parallel schedules) and the Table 7 statistics.  Validates ids
+ *   (UG_ERR_INDEX_RANGE).  May synchronise `stream`.  *out owns copies of everything.
+ */
+ug_status ug_graph_create(int64_t num_vertices, int64_t num_edges,
+                          const int32_t *src, const int32_t *dst, int on_device, int flags,
+                          const ug_allocator *alloc, void *stream, ug_graph **out);
+
+/* CSR input: row_ptr[V+1] (non-decreasing, row_ptr[0] = 0, row_ptr[V] = E), col_idx[E] = src,
+ * eid[E] = COO edge id of CSR position k (NULL = identity).  Host or device per on_device. */
+ug_status ug_graph_create_csr(int64_t num_vertices, int64_t num_edges, const int32_t *row_ptr,
+                              const int32_t *col_idx, const int32_t *eid, int on_device, int flags,
+                              const ug_allocator *alloc, void *stream, ug_graph **out);
+
+/* Frees a graph or a view.  A parent must outlive its views. */
+ug_status ug_graph_destroy(ug_graph *g);
+
+/* Table 7 graph features: V (dst rows), E, mean in-degree,
+ * std_nnz = population std of in-degree (R15), max in-degree.  Any out pointer may be NULL. */
+ug_status ug_graph_stats(const ug_graph *g, int64_t *V, int64_t *E, double *mean_deg,
+                         double *std_nnz, int64_t *max_deg);
+
+/* Copy the host CSR (row_ptr[V+1], col_idx[E], eid[E]) into caller buffers (any may be NULL). */
+ug_status ug_graph_csr(const ug_graph *g, int32_t *row_ptr, int32_t *col_idx, int32_t *eid);
+
+/* Edge-balanced destination-row partition (R21): row_splits[k] = smallest row r with
+ * row_ptr[r] >= ceil(k E / parts), row_splits[0] = 0, row_splits[parts] = V. */
+ug_status ug_graph_partition(const ug_graph *g, int32_t parts, int64_t *row_splits);
+
+/*
+ * ug_graph_view_rows -- zero-copy view of destination rows [r0, r1) for sharding.
+ *   Inside a view: Src_V operands are indexed by GLOBAL vertex id (pass the full,
+ *   all-gathered X); Dst_V operands and C of type Dst_V by LOCAL row v - r0 (pass
+ *   X_full + r0*ld and the local output shard); Edge operands and C of type Edge by LOCAL
+ *   edge position k - row_ptr[r0].  Requires eid = identity (dst-sorted COO); otherwise
+ *   UG_ERR_INVALID_ARG (permute edge tensors once with ug_edge_permute).
+ */
+ug_status ug_graph_view_rows(const ug_graph *g, int64_t r0, int64_t r1, ug_graph **view);
+
+/* Validate op_info against the supported op set and shapes without running (host only). */
+ug_status ug_op_validate(const ug_graph *g, const ug_op_info *op);
+
+/*
+ * ug_schedule_select -- automatic choice of parallel_info when it is absent.
+ * Keyed by (op class, F, mean degree, degree CV, V) over a table measured on B200
+ * (selector_table.json, loaded at first use or via ug_selector_load).  Host only, < 10 us.
+ */
+ug_status ug_schedule_select(const ug_graph *g, const ug_op_info *op, ug_schedule *out);
+
+/* Replace the selector table with the JSON file at `path` (format in DESIGN.md). */
+ug_status ug_selector_load(const char *path);
+
+/*
+ * ug_op_run -- one unified-operator call (the paper's uGrapher(Graph_Tensor, op_info,
+ * parallel_info)).  sched NULL or strategy UG_SCHED_AUTO -> ug_schedule_select.
+ * Writes every element of C's logical [rows x width] block (rows with zero in-degree get
+ * 0, R7).  Enqueues 1-3 kernels on `stream` (init / main / epilogue as the schedule needs);
+ * never synchronises.  Requires a device graph (not UG_GRAPH_HOST_ONLY).
+ */
+ug_status ug_op_run(const ug_graph *g, const ug_op_info *op, const ug_schedule *sched,
+                    void *stream);
+
+/* Measurement hook: exactly ug_op_run, and additionally records the caller's cudaEvent_t
+ * `ev_begin` / `ev_end` on `stream` immediately before / after the operator's MAIN kernel
+ * (the traversal a5, excluding init / epilogue / fix-up launches), so a caller can time the
+ * dominant kernel alone with CUDA events.  Either event may be NULL. */
+ug_status ug_op_run_events(const ug_graph *g, const ug_op_info *op, const ug_schedule *sched,
+                           void *stream, void *ev_begin, void *ev_end);
+
+/* Number of kernel launches ug_op_run would enqueue for (op, sched) (after AUTO). */
+ug_status ug_op_launch_count(const ug_graph *g, const ug_op_info *op, const ug_schedule *sched,
+                             int32_t *launches);
+
+/* out[k][:] = in[eid[k]][:] for k < E: edge tensor from COO edge-id order to CSR order
+ * (device pointers, width columns, dense rows).  Identity copy when eid is identity. */
+ug_status ug_edge_permute(const ug_graph *g, const float *in, float *out, int32_t width,
+                          void *stream);
+
+/* Schedule <-> text, Table 9 notation ("TE_G1_T16", "SV_G2048_F64"). */
+ug_status ug_schedule_parse(const char *text, ug_schedule *out);
+ug_status ug_schedule_format(const ug_schedule *s, char *buf, size_t len);
+
+const char *ug_status_string(ug_status s);
+const char *ug_last_error(void);   /* thread-local detail of the last failing call */
+const char *ug_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* UG_H_ */

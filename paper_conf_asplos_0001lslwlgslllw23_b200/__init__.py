@@ -1,0 +1,237 @@
+"""ugraph-b200: the unified GNN graph operator of uGrapher (ASPLOS'23) on B200 (sm_100a).
+
+Thin Python binding over the C ABI in include/ug.h (libugraph.so).  Everything here is
+argument marshalling: torch supplies device memory and the current stream; every step of
+the operator runs in the library's CUDA kernels.  There is no CPU fallback.
+
+    g = Graph(V, src, dst)                         # ug_graph_create (COO -> in-CSR)
+    op_run(g, "mul", "sum", A=X, a_type="u", B=w, b_type="e", C=Y, c_type="v")
+                                                   # uGrapher(graph, op_info, parallel_info)
+    schedule_select(g, ...)                        # parallel_info when absent
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+
+from . import _ffi
+from ._ffi import (EDGE_OPS, GATHER_OPS, STRATEGIES, TTYPES, UgError, UgOpInfo, UgSchedule,
+                   UgTensor, check, lib)
+
+__all__ = ["Graph", "op_run", "schedule_select", "launch_count", "parse_schedule",
+           "format_schedule", "validate", "edge_permute", "selector_load", "UgError", "version"]
+
+
+def version():
+    return lib.ug_version().decode()
+
+
+def _current_stream(stream):
+    if stream is not None:
+        return ctypes.c_void_p(int(stream))
+    import torch
+    if torch.cuda.is_available():
+        return ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    return ctypes.c_void_p(0)
+
+
+def _int32_buffer(x):
+    """(pointer, on_device, keepalive) for an int32 array (numpy or torch, host or CUDA)."""
+    try:
+        import torch
+        if isinstance(x, torch.Tensor):
+            if x.dtype != torch.int32:
+                raise TypeError("index tensors must be int32")
+            x = x.contiguous()
+            return x.data_ptr(), int(x.is_cuda), x
+    except ImportError:
+        pass
+    a = np.ascontiguousarray(x, dtype=np.int32)
+    return a.ctypes.data, 0, a
+
+
+class Graph:
+    """A destination-keyed CSR graph owned by libugraph (ug_graph)."""
+
+    def __init__(self, num_vertices, src=None, dst=None, *, host_only=False, stream=None, _handle=None,
+                 _parent=None):
+        self._parent = _parent
+        if _handle is not None:
+            self._h = _handle
+            return
+        sp, sdev, ka = _int32_buffer(src)
+        dp, ddev, kb = _int32_buffer(dst)
+        if sdev != ddev:
+            raise ValueError("src and dst must both be host or both device arrays")
+        E = int(ka.shape[0])
+        h = ctypes.c_void_p()
+        flags = _ffi.UG_GRAPH_HOST_ONLY if host_only else 0
+        st = lib.ug_graph_create(int(num_vertices), E, sp, dp, sdev, flags, None,
+                                 None if host_only else _current_stream(stream), ctypes.byref(h))
+        check(st, "ug_graph_create")
+        self._h = h
+
+    @classmethod
+    def from_csr(cls, num_vertices, row_ptr, col_idx, eid=None, *, host_only=False, stream=None):
+        rp, rdev, ka = _int32_buffer(row_ptr)
+        cp, cdev, kb = _int32_buffer(col_idx)
+        ep, kc = (None, None)
+        if eid is not None:
+            ep, _, kc = _int32_buffer(eid)
+        h = ctypes.c_void_p()
+        flags = _ffi.UG_GRAPH_HOST_ONLY if host_only else 0
+        st = lib.ug_graph_create_csr(int(num_vertices), int(kb.shape[0]), rp, cp, ep, rdev, flags, None,
+                                     None if host_only else _current_stream(stream), ctypes.byref(h))
+        check(st, "ug_graph_create_csr")
+        return cls(num_vertices, _handle=h)
+
+    @property
+    def handle(self):
+        return self._h
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value:
+            lib.ug_graph_destroy(h)
+            self._h = None
+
+    def stats(self):
+        V, E, mx = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+        mean, std = ctypes.c_double(), ctypes.c_double()
+        check(lib.ug_graph_stats(self._h, ctypes.byref(V), ctypes.byref(E), ctypes.byref(mean),
+                                 ctypes.byref(std), ctypes.byref(mx)), "ug_graph_stats")
+        return {"V": V.value, "E": E.value, "mean_deg": mean.value, "std_nnz": std.value,
+                "max_deg": mx.value}
+
+    @property
+    def num_rows(self):
+        return self.stats()["V"]
+
+    @property
+    def num_edges(self):
+        return self.stats()["E"]
+
+    def csr(self):
+        s = self.stats()
+        rp = np.zeros(s["V"] + 1, np.int32)
+        col = np.zeros(max(s["E"], 1), np.int32)
+        eid = np.zeros(max(s["E"], 1), np.int32)
+        check(lib.ug_graph_csr(self._h, rp.ctypes.data, col.ctypes.data, eid.ctypes.data), "ug_graph_csr")
+        return rp, col[:s["E"]], eid[:s["E"]]
+
+    def partition(self, parts):
+        out = np.zeros(parts + 1, np.int64)
+        check(lib.ug_graph_partition(self._h, int(parts), out.ctypes.data), "ug_graph_partition")
+        return out
+
+    def view_rows(self, r0, r1):
+        h = ctypes.c_void_p()
+        check(lib.ug_graph_view_rows(self._h, int(r0), int(r1), ctypes.byref(h)), "ug_graph_view_rows")
+        return Graph(0, _handle=h, _parent=self)
+
+
+def _tensor(x, ttype, rows_hint=None):
+    if x is None:
+        return UgTensor(None, TTYPES[None], 0, 0)
+    import torch
+    if not isinstance(x, torch.Tensor):
+        raise TypeError("operands must be torch tensors on the CUDA device")
+    if x.dtype != torch.float32:
+        raise TypeError("operands must be float32")
+    if x.dim() == 1:
+        x = x.view(-1, 1)
+    if x.dim() != 2 or x.stride(1) != 1:
+        raise ValueError("operands must be 2-D with unit column stride")
+    return UgTensor(x.data_ptr(), TTYPES[ttype], x.shape[1], max(x.stride(0), x.shape[1]))
+
+
+def _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H):
+    if F is None:
+        ref = A if A is not None else B
+        F = ref.shape[1] if ref.dim() == 2 else 1
+        if edge_op == "dot" and C is not None and H is None:
+            H = C.shape[1] if C.dim() == 2 else 1
+    if H is None:
+        H = 1
+    return UgOpInfo(EDGE_OPS[edge_op], GATHER_OPS[gather_op], _tensor(A, a_type), _tensor(B, b_type),
+                    _tensor(C, c_type), int(F), int(H))
+
+
+def parse_schedule(text):
+    s = UgSchedule()
+    check(lib.ug_schedule_parse(text.encode(), ctypes.byref(s)), f"ug_schedule_parse({text})")
+    return s
+
+
+def format_schedule(s):
+    buf = ctypes.create_string_buffer(64)
+    check(lib.ug_schedule_format(ctypes.byref(s), buf, 64), "ug_schedule_format")
+    return buf.value.decode()
+
+
+def _sched(schedule):
+    if schedule is None:
+        return None
+    if isinstance(schedule, UgSchedule):
+        return ctypes.byref(schedule)
+    return ctypes.byref(parse_schedule(schedule))
+
+
+def op_run(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, C=None, c_type="v",
+           F=None, H=None, schedule=None, stream=None):
+    """One unified-operator call (uGrapher(Graph_Tensor, op_info, parallel_info)).
+
+    A, B, C: CUDA float32 tensors [rows, width] (row stride may exceed width); types are
+    "u" (Src_V), "v" (Dst_V), "e" (Edge) or None.  C is written in place.  schedule: None
+    (automatic) or Table 9 notation such as "TE_G1_T16" / "SV_G2048_F64".
+    Asynchronous on `stream` (default: torch's current stream).
+    """
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+    check(lib.ug_op_run(graph.handle, ctypes.byref(info), _sched(schedule), _current_stream(stream)),
+          "ug_op_run")
+    return C
+
+
+def op_run_events(graph, edge_op, gather_op, ev_begin, ev_end, A=None, a_type=None, B=None, b_type=None,
+                  C=None, c_type="v", F=None, H=None, schedule=None, stream=None):
+    """op_run that also records torch.cuda.Event pair (ev_begin, ev_end) around the main kernel
+    (measurement hook, ug_op_run_events).  The events must have been recorded once before."""
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+    check(lib.ug_op_run_events(graph.handle, ctypes.byref(info), _sched(schedule), _current_stream(stream),
+                               ctypes.c_void_p(ev_begin.cuda_event), ctypes.c_void_p(ev_end.cuda_event)),
+          "ug_op_run_events")
+    return C
+
+
+def validate(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, C=None, c_type="v",
+             F=None, H=None):
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+    check(lib.ug_op_validate(graph.handle, ctypes.byref(info)), "ug_op_validate")
+
+
+def schedule_select(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, C=None,
+                    c_type="v", F=None, H=None):
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+    s = UgSchedule()
+    check(lib.ug_schedule_select(graph.handle, ctypes.byref(info), ctypes.byref(s)), "ug_schedule_select")
+    return format_schedule(s)
+
+
+def launch_count(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, C=None, c_type="v",
+                 F=None, H=None, schedule=None):
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+    n = ctypes.c_int32()
+    check(lib.ug_op_launch_count(graph.handle, ctypes.byref(info), _sched(schedule), ctypes.byref(n)),
+          "ug_op_launch_count")
+    return n.value
+
+
+def edge_permute(graph, inp, out, stream=None):
+    check(lib.ug_edge_permute(graph.handle, inp.data_ptr(), out.data_ptr(), inp.shape[1],
+                              _current_stream(stream)), "ug_edge_permute")
+    return out
+
+
+def selector_load(path):
+    check(lib.ug_selector_load(str(path).encode()), "ug_selector_load")

@@ -1,0 +1,182 @@
+// k_common.cuh -- device functions shared by the schedule templates (the paper's
+// "device function interface": global-function templates per strategy,
+// device functions per arithmetic).  Compiled with -fmad=true but every message is formed
+// with explicit _rn intrinsics so it is rounded once, exactly as a standalone
+// message-creation op would (reading R11); accumulation order is the only freedom.
+#pragma once
+#include <cuda_runtime.h>
+#include <math_constants.h>
+#include <stdint.h>
+
+#include "ug_internal.h"
+
+namespace ug {
+
+// ---------------------------------------------------------------- edge_op (Fig. 5 line 18)
+template <int KE>
+__device__ __forceinline__ float edge_fn(float a, float b) {
+    if constexpr (KE == K_COPY) return a;
+    else if constexpr (KE == K_ADD) return __fadd_rn(a, b);
+    else if constexpr (KE == K_SUB) return __fsub_rn(a, b);
+    else if constexpr (KE == K_MUL) return __fmul_rn(a, b);
+    else return __fdiv_rn(a, b);
+}
+
+// ---------------------------------------------------------------- gather_op (Fig. 5 line 19)
+// Total order with -0 < +0 (R12): fmaxf/fminf plus an explicit tie rule for +-0.
+__device__ __forceinline__ float tmax(float a, float b) {
+    float m = fmaxf(a, b);
+    if (a == b) m = __int_as_float(__float_as_int(a) & __float_as_int(b));
+    return m;
+}
+__device__ __forceinline__ float tmin(float a, float b) {
+    float m = fminf(a, b);
+    if (a == b) m = __int_as_float(__float_as_int(a) | __float_as_int(b));
+    return m;
+}
+
+template <int GOP>
+__device__ __forceinline__ float g_init() {
+    if constexpr (GOP == UG_GATHER_MAX) return -CUDART_INF_F;
+    else if constexpr (GOP == UG_GATHER_MIN) return CUDART_INF_F;
+    else return 0.0f;
+}
+
+template <int GOP>
+__device__ __forceinline__ float g_combine(float acc, float m) {
+    if constexpr (GOP == UG_GATHER_MAX) return tmax(acc, m);
+    else if constexpr (GOP == UG_GATHER_MIN) return tmin(acc, m);
+    else return __fadd_rn(acc, m);
+}
+
+// Final value of an owner-computed row (R7 zero in-degree -> 0; R8 mean = sum / deg with one
+// IEEE division).
+template <int GOP>
+__device__ __forceinline__ float g_finalize(float acc, int64_t deg) {
+    if (deg == 0) return 0.0f;
+    if constexpr (GOP == UG_GATHER_MEAN) return __fdiv_rn(acc, (float)deg);
+    else return acc;
+}
+
+// ---------------------------------------------------------------- vector loads
+template <int VEC> struct VecT;
+template <> struct VecT<1> { using T = float; };
+template <> struct VecT<2> { using T = float2; };
+template <> struct VecT<4> { using T = float4; };
+
+template <int VEC>
+__device__ __forceinline__ void ldg_vec(const float *__restrict__ p, float (&r)[VEC]) {
+    if constexpr (VEC == 1) {
+        r[0] = __ldg(p);
+    } else if constexpr (VEC == 2) {
+        float2 t = __ldg(reinterpret_cast<const float2 *>(p));
+        r[0] = t.x; r[1] = t.y;
+    } else {
+        float4 t = __ldg(reinterpret_cast<const float4 *>(p));
+        r[0] = t.x; r[1] = t.y; r[2] = t.z; r[3] = t.w;
+    }
+}
+
+template <int VEC>
+__device__ __forceinline__ void st_vec(float *p, const float (&r)[VEC]) {
+    if constexpr (VEC == 1) {
+        p[0] = r[0];
+    } else if constexpr (VEC == 2) {
+        *reinterpret_cast<float2 *>(p) = make_float2(r[0], r[1]);
+    } else {
+        *reinterpret_cast<float4 *>(p) = make_float4(r[0], r[1], r[2], r[3]);
+    }
+}
+
+// Store the first n (<= VEC) lanes of a vector: the ragged tail of a row.
+template <int VEC>
+__device__ __forceinline__ void st_vec_n(float *p, const float (&r)[VEC], int n) {
+    if (n >= VEC) { st_vec<VEC>(p, r); return; }
+#pragma unroll
+    for (int i = 0; i < VEC; ++i)
+        if (i < n) p[i] = r[i];
+}
+
+// Row of an operand for the edge (src, dst, e): type_idx_dict.
+__device__ __forceinline__ int64_t op_row(int32_t type, int64_t src, int64_t dst, int64_t e) {
+    return type == UG_T_SRC_V ? src : (type == UG_T_DST_V ? dst : e);
+}
+
+// Column of feature f in an operand: full width -> f, per-head width -> f / D (R6).
+__device__ __forceinline__ int64_t op_col(const Operand &x, int f) {
+    return x.div == 1 ? (int64_t)f : (int64_t)(f / x.div);
+}
+
+// VEC features starting at column `col` of row `row` (broadcast when x.div > 1; the
+// VEC features of one chunk always lie inside one head: the host guarantees D % VEC == 0).
+template <int VEC>
+__device__ __forceinline__ void fetch(const Operand &x, int64_t row, int64_t col, float (&r)[VEC]) {
+    const float *p = x.p + row * x.ld + col;
+    if (x.div == 1) {
+        ldg_vec<VEC>(p, r);
+    } else {
+        float s = __ldg(p);
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) r[i] = s;
+    }
+}
+
+// Message vector for one edge (elementwise ops).
+template <int KE, int VEC>
+__device__ __forceinline__ void message(const OpArgs &op, int64_t ra, int64_t ca, int64_t rb,
+                                        int64_t cb, float (&m)[VEC]) {
+    float a[VEC];
+    fetch<VEC>(op.A, ra, ca, a);
+    if constexpr (KE == K_COPY) {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) m[i] = a[i];
+    } else {
+        float b[VEC];
+        fetch<VEC>(op.B, rb, cb, b);
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) m[i] = edge_fn<KE>(a[i], b[i]);
+    }
+}
+
+// ---------------------------------------------------------------- atomics (pass 2)
+// max/min on fp32 by the integer-order trick: non-negative floats order like signed ints,
+// negative floats order reversed as unsigned ints; -0 (0x80000000) < +0 (0).
+__device__ __forceinline__ void atomic_max_f32(float *addr, float v) {
+    if (!signbit(v)) atomicMax(reinterpret_cast<int *>(addr), __float_as_int(v));
+    else atomicMin(reinterpret_cast<unsigned int *>(addr), __float_as_uint(v));
+}
+__device__ __forceinline__ void atomic_min_f32(float *addr, float v) {
+    if (!signbit(v)) atomicMin(reinterpret_cast<int *>(addr), __float_as_int(v));
+    else atomicMax(reinterpret_cast<unsigned int *>(addr), __float_as_uint(v));
+}
+
+template <int GOP, int VEC>
+__device__ __forceinline__ void atomic_flush(float *p, const float (&acc)[VEC], int n) {
+    if constexpr (GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN) {
+        if (n >= VEC) {
+            if constexpr (VEC == 4) {
+                atomicAdd(reinterpret_cast<float4 *>(p), make_float4(acc[0], acc[1], acc[2], acc[3]));
+                return;
+            } else if constexpr (VEC == 2) {
+                atomicAdd(reinterpret_cast<float2 *>(p), make_float2(acc[0], acc[1]));
+                return;
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < VEC; ++i)
+            if (i < n) atomicAdd(p + i, acc[i]);
+    } else {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) {
+            if (i < n) {
+                if constexpr (GOP == UG_GATHER_MAX) atomic_max_f32(p + i, acc[i]);
+                else atomic_min_f32(p + i, acc[i]);
+            }
+        }
+    }
+}
+
+// Helpers for launch sizing.
+__host__ __device__ __forceinline__ int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+}  // namespace ug

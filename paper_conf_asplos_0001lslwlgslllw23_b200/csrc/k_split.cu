@@ -1,0 +1,141 @@
+// k_split.cu -- Split-Vertex (SV), the B200 schedule for wide, skewed aggregations
+// (C3/C5).  It composes the paper's two knobs with two B200 facts: a
+// 126 MB L2 and 148 SMs that all want equal work.
+//
+//  * Row splitting (load balance): every destination row is cut into chunks of at most
+//    `group` in-edges (a hub of in-degree 4.9e4 becomes ~24 chunks).  A chunk is one work
+//    unit; rows with one chunk are owned and finalised in registers; the partial results
+//    of split rows go to a scratch slot and a fix-up kernel combines them in chunk order
+//    (deterministic; no atomics, no init pass).
+//  * Column tiles, tile-major (locality): the feature axis is cut into ftile-wide tiles and
+//    the grid is ordered tile-major, so at any time the gathered rows touch one
+//    V x ftile slab of X (C5, ftile 64: 60 MB) which stays L2-resident while the next
+//    slab streams in; each X element then comes from DRAM about once per tile pass
+//    instead of once per in-edge.
+//  * L = ftile / VEC lanes per unit (one VEC-wide feature chunk per lane), the in-edge loop
+//    unrolled 4x so each lane keeps 4 independent row gathers in flight.
+#include "k_dispatch.cuh"
+
+namespace ug {
+
+template <int KE, int GOP, int VEC>
+__global__ void __launch_bounds__(256) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
+                                               int64_t n_chunks, int L_log2, int ftile, int n_tiles,
+                                               float *__restrict__ scratch, int64_t sld) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int lane = (int)(t & ((1 << L_log2) - 1));
+    const int64_t u = t >> L_log2;
+    if (u >= n_chunks * n_tiles) return;
+    const int tile = (int)(u / n_chunks);
+    const int64_t c = u - (int64_t)tile * n_chunks;
+    const int f = tile * ftile + lane * VEC;
+    if (f >= op.W) return;
+    const int4 ch = chunks[c];
+    const int64_t v = ch.x;
+    const int64_t k1 = ch.z;
+    const int64_t ca = op_col(op.A, f);
+    const int64_t cb = op_col(op.B, f);
+
+    if constexpr (GOP == UG_GATHER_ASSIGN) {
+        for (int64_t k = ch.y; k < k1; ++k) {
+            const int64_t src = g.col[k];
+            const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
+            float m[VEC];
+            message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m);
+            st_vec_n<VEC>(op.C + e * op.c_ld + f, m, op.W - f);
+        }
+    } else {
+        float acc[VEC];
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) acc[i] = g_init<GOP>();
+        int64_t k = ch.y;
+        for (; k + 4 <= k1; k += 4) {
+            float m[4][VEC];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int64_t src = g.col[k + q];
+                const int64_t e = g.eid ? (int64_t)g.eid[k + q] : k + q;
+                message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m[q]);
+            }
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[q][i]);
+        }
+        for (; k < k1; ++k) {
+            const int64_t src = g.col[k];
+            const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
+            float m[VEC];
+            message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m);
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[i]);
+        }
+        if (ch.w < 0) {
+            const int64_t deg = (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
+            float out[VEC];
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) out[i] = g_finalize<GOP>(acc[i], deg);
+            st_vec_n<VEC>(op.C + v * op.c_ld + f, out, op.W - f);
+        } else {
+            st_vec<VEC>(scratch + (int64_t)ch.w * sld + f, acc);
+        }
+    }
+}
+
+// Fix-up of split rows: combine the row's partials in chunk order, finalise, store.
+template <int GOP, int VEC>
+__global__ void k_split_fix(GraphArgs g, OpArgs op, const int4 *__restrict__ split, int64_t n_split,
+                            const float *__restrict__ scratch, int64_t sld) {
+    const int64_t per_row = cdiv(op.W, VEC);
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= n_split * per_row) return;
+    const int64_t r = t / per_row;
+    const int f = (int)(t - r * per_row) * VEC;
+    const int4 sp = split[r];
+    float acc[VEC];
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) acc[i] = g_init<GOP>();
+    for (int s = 0; s < sp.z; ++s) {
+        float p[VEC];
+        ldg_vec<VEC>(scratch + (int64_t)(sp.y + s) * sld + f, p);
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], p[i]);
+    }
+    const int64_t v = sp.x;
+    const int64_t deg = (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) acc[i] = g_finalize<GOP>(acc[i], deg);
+    st_vec_n<VEC>(op.C + v * op.c_ld + f, acc, op.W - f);
+}
+
+cudaError_t launch_split_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
+                                const LaunchCfg &c, const SplitPlan &plan, float *scratch,
+                                cudaStream_t s, cudaEvent_t ev_begin, cudaEvent_t ev_end) {
+    const int L = c.ftile / c.vec;
+    const int n_tiles = (int)cdiv(op.W, c.ftile);
+    const int64_t threads = plan.n_chunks * n_tiles * (int64_t)L;
+    if (threads == 0) return cudaSuccess;
+    const int64_t grid = cdiv(threads, c.block);
+    const int L_log2 = ilog2(L);
+    const int64_t sld = cdiv(op.W, 4) * 4;
+    const int4 *chunks = reinterpret_cast<const int4 *>(plan.d_chunk);
+    if (ev_begin) cudaEventRecord(ev_begin, s);
+    UG_DISPATCH_VEC(c.vec, VEC,
+        UG_DISPATCH_KE(kedge, KE,
+            UG_DISPATCH_GOP(gather, GOP,
+                k_split<KE, GOP, VEC><<<(unsigned)grid, c.block, 0, s>>>(
+                    g, op, chunks, plan.n_chunks, L_log2, c.ftile, n_tiles, scratch, sld))));
+    if (ev_end) cudaEventRecord(ev_end, s);
+    cudaError_t err = cudaGetLastError();
+    if (err != cudaSuccess || gather == UG_GATHER_ASSIGN || plan.n_split_rows == 0) return err;
+    const int64_t per_row = cdiv(op.W, c.vec);
+    const int64_t fgrid = cdiv(plan.n_split_rows * per_row, 256);
+    const int4 *split = reinterpret_cast<const int4 *>(plan.d_split);
+    UG_DISPATCH_VEC(c.vec, VEC,
+        UG_DISPATCH_RED(gather, GOP,
+            k_split_fix<GOP, VEC><<<(unsigned)fgrid, 256, 0, s>>>(g, op, split, plan.n_split_rows,
+                                                                  scratch, sld)));
+    return cudaGetLastError();
+}
+
+}  // namespace ug

@@ -1,0 +1,116 @@
+// k_vertex.cu -- vertex-parallel owner-computes template: Thread-Vertex and Warp-Vertex
+// (Fig. 6(b),(d)) with V-grouping G and feature
+// tiling T (Fig. 6(f)).
+//
+// Canonical form: a unit is one destination row; L lanes share the
+// unit's features (TV: L = T threads, WV: L = 32 T); lane l owns the VEC-wide feature
+// chunks l, l + L, l + 2L, ... (Fig. 6(f): f = f10*32*T + f11*32 + f2).  A lane group
+// processes G consecutive rows.  Rows are owned: no atomics, mean / zero-degree handled in
+// registers (pass 2 of PAPER.md:405 inserts no atomics here).  With ftile > 0 the feature
+// axis is first cut into column tiles ordered tile-major over the grid, so the rows being
+// gathered concurrently touch one ftile-wide column slab of the operands (L2 residency).
+// With C = Edge (message creation) the same traversal writes each in-edge's message.
+#include "k_dispatch.cuh"
+
+namespace ug {
+
+template <int KE, int GOP, int VEC>
+__global__ void __launch_bounds__(256) k_vertex(GraphArgs g, OpArgs op, int L_log2, int G,
+                                                int ftile, int64_t n_groups, int n_tiles) {
+    constexpr int R = (8 / VEC) > 0 ? (8 / VEC) : 1;   // register chunks per lane (8 floats)
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int L = 1 << L_log2;
+    const int lane = (int)(t & (L - 1));
+    const int64_t grp = t >> L_log2;
+    if (grp >= n_groups * n_tiles) return;
+    const int tile = (int)(grp / n_groups);
+    const int64_t ugp = grp - (int64_t)tile * n_groups;
+    const int f_lo = tile * ftile;
+    const int f_hi = min(op.W, f_lo + ftile);
+    const int stride = L * VEC;
+    const int64_t v_end = min(g.V, (ugp + 1) * (int64_t)G);
+
+    for (int64_t v = ugp * (int64_t)G; v < v_end; ++v) {
+        const int64_t k0 = (int64_t)g.row_ptr[v] - g.rp_base;
+        const int64_t k1 = (int64_t)g.row_ptr[v + 1] - g.rp_base;
+        for (int fb = f_lo + lane * VEC; fb < f_hi; fb += stride * R) {
+            int64_t ca[R], cb[R];
+#pragma unroll
+            for (int j = 0; j < R; ++j) {
+                const int f = fb + j * stride;
+                ca[j] = op_col(op.A, f);
+                cb[j] = op_col(op.B, f);
+            }
+            if constexpr (GOP == UG_GATHER_ASSIGN) {
+                for (int64_t k = k0; k < k1; ++k) {
+                    const int64_t src = g.col[k];
+                    const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
+                    const int64_t ra = op_row(op.A.type, src, v, e);
+                    const int64_t rb = op_row(op.B.type, src, v, e);
+#pragma unroll
+                    for (int j = 0; j < R; ++j) {
+                        const int f = fb + j * stride;
+                        if (f < f_hi) {
+                            float m[VEC];
+                            message<KE, VEC>(op, ra, ca[j], rb, cb[j], m);
+                            st_vec_n<VEC>(op.C + e * op.c_ld + f, m, op.W - f);
+                        }
+                    }
+                }
+            } else {
+                float acc[R][VEC];
+#pragma unroll
+                for (int j = 0; j < R; ++j)
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) acc[j][i] = g_init<GOP>();
+                for (int64_t k = k0; k < k1; ++k) {
+                    const int64_t src = g.col[k];
+                    const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
+                    const int64_t ra = op_row(op.A.type, src, v, e);
+                    const int64_t rb = op_row(op.B.type, src, v, e);
+#pragma unroll
+                    for (int j = 0; j < R; ++j) {
+                        const int f = fb + j * stride;
+                        if (f < f_hi) {
+                            float m[VEC];
+                            message<KE, VEC>(op, ra, ca[j], rb, cb[j], m);
+#pragma unroll
+                            for (int i = 0; i < VEC; ++i) acc[j][i] = g_combine<GOP>(acc[j][i], m[i]);
+                        }
+                    }
+                }
+                const int64_t deg = k1 - k0;
+#pragma unroll
+                for (int j = 0; j < R; ++j) {
+                    const int f = fb + j * stride;
+                    if (f < f_hi) {
+                        float out[VEC];
+#pragma unroll
+                        for (int i = 0; i < VEC; ++i) out[i] = g_finalize<GOP>(acc[j][i], deg);
+                        st_vec_n<VEC>(op.C + v * op.c_ld + f, out, op.W - f);
+                    }
+                }
+            }
+        }
+    }
+}
+
+cudaError_t launch_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
+                          const LaunchCfg &c, cudaStream_t s) {
+    const int ft = c.ftile > 0 ? c.ftile : op.W;
+    const int n_tiles = (int)cdiv(op.W, ft);
+    const int64_t n_groups = cdiv(g.V, c.G);
+    const int64_t threads = n_groups * n_tiles * (int64_t)c.L;
+    if (threads == 0) return cudaSuccess;
+    const int block = c.block;
+    const int64_t grid = cdiv(threads, block);
+    const int L_log2 = ilog2(c.L);
+    UG_DISPATCH_VEC(c.vec, VEC,
+        UG_DISPATCH_KE(kedge, KE,
+            UG_DISPATCH_GOP(gather, GOP,
+                k_vertex<KE, GOP, VEC><<<(unsigned)grid, block, 0, s>>>(g, op, L_log2, c.G, ft,
+                                                                        n_groups, n_tiles))));
+    return cudaGetLastError();
+}
+
+}  // namespace ug

@@ -1,0 +1,119 @@
+// ug_internal.h -- runtime <-> kernel interface of libugraph (not part of the C ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <map>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "ug.h"
+
+namespace ug {
+
+// Operand as the kernels see it (PAPER.md:232 type_idx_dict + head broadcast, R6).
+struct Operand {
+    const float *p;   // base pointer (already offset for views where needed)
+    int32_t type;     // UG_T_*
+    int32_t div;      // F / width: 1 = full width, D = per-head broadcast, F = scalar
+    int64_t ld;       // row stride (elements)
+};
+
+// CSR view as the kernels see it.  Positions k are LOCAL: k in [0, E).
+struct GraphArgs {
+    const int32_t *row_ptr;  // row_ptr[v] - rp_base = first local position of local row v
+    const int32_t *col;      // col[k]  = global src id of local position k
+    const int32_t *eid;      // eid[k]  = edge id of position k (NULL = identity)
+    const int32_t *dst;      // dst[k]  = GLOBAL dst row of position k (edge-parallel schedules)
+    int64_t V;               // local rows
+    int64_t E;               // local edges
+    int64_t rp_base;         // row_ptr[r0] of a view (0 for a base graph)
+    int64_t r0;              // first global row of a view (0 for a base graph)
+};
+
+struct OpArgs {
+    Operand A, B;
+    float *C;
+    int64_t c_ld;
+    int32_t c_type;   // UG_T_DST_V (aggregate) or UG_T_EDGE (message creation)
+    int32_t F;        // feature width
+    int32_t W;        // message / output width (F, or H for dot)
+    int32_t H, D;     // heads, D = F / H
+};
+
+// Normalised edge ops inside the kernels (copy_rhs is rewritten as copy_lhs on B).
+enum KEdge { K_COPY = 0, K_ADD = 1, K_SUB = 2, K_MUL = 3, K_DIV = 4 };
+
+struct LaunchCfg {
+    int strategy;     // UG_TV ... UG_SV
+    int L;            // lanes per unit (power of two)
+    int G;            // units per lane group (or chunk size for SV)
+    int block;        // CTA size
+    int ftile;        // column tile width (multiple of vec), 0 = whole width
+    int vec;          // 1, 2, 4
+};
+
+// Split-row plan for UG_SV (built once per (graph, chunk size), cached on the graph).
+struct SplitPlan {
+    int64_t n_chunks = 0;       // work units per column tile
+    int64_t n_split_rows = 0;   // rows cut into >1 chunk
+    int64_t n_split_chunks = 0; // chunks belonging to split rows (scratch slots)
+    int32_t *d_chunk = nullptr;   // [n_chunks] x 4 int32: row, k0, k1, scratch slot (-1 = owner)
+    int32_t *d_split = nullptr;   // [n_split_rows] x 4 int32: row, first slot, n slots, 0
+};
+
+// Kernel launchers (kernels/*.cu).  All return cudaGetLastError().
+cudaError_t launch_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
+                          const LaunchCfg &c, cudaStream_t s);
+cudaError_t launch_edge(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
+                        const LaunchCfg &c, cudaStream_t s);
+cudaError_t launch_block_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
+                                const LaunchCfg &c, cudaStream_t s);
+cudaError_t launch_split_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
+                                const LaunchCfg &c, const SplitPlan &plan, float *scratch,
+                                cudaStream_t s, cudaEvent_t ev_begin = nullptr, cudaEvent_t ev_end = nullptr);
+cudaError_t launch_dot(bool vertex_units, int gather, const GraphArgs &g, const OpArgs &op,
+                       const LaunchCfg &c, cudaStream_t s);
+cudaError_t launch_init(int gather, const OpArgs &op, int64_t rows, cudaStream_t s);
+cudaError_t launch_epilogue(int gather, const GraphArgs &g, const OpArgs &op, cudaStream_t s);
+cudaError_t launch_permute(const int32_t *eid, const float *in, float *out, int64_t E, int width,
+                           cudaStream_t s);
+
+}  // namespace ug
+
+// The opaque graph of the C ABI.
+struct ug_graph {
+    int64_t V = 0, E = 0;       // local rows / edges
+    int64_t V_total = 0;        // vertex-id space (src ids < V_total)
+    int64_t r0 = 0;             // first global row (views)
+    int64_t e0 = 0;             // first global CSR position (views) == row_ptr[r0]
+    bool host_only = false;
+    bool is_view = false;
+    bool eid_identity = true;
+    const ug_graph *parent = nullptr;
+
+    // Host CSR.  Base graphs own the vectors; views point into the parent's arrays.
+    std::vector<int32_t> h_row_ptr_v, h_col_v, h_eid_v, h_dst_v;
+    const int32_t *h_row_ptr = nullptr;   // global row_ptr values at local rows 0..V
+    const int32_t *h_col = nullptr;       // at local position 0
+    const int32_t *h_eid = nullptr;       // NULL when identity
+
+    // Device CSR (same offsets as the host pointers).
+    int32_t *d_row_ptr = nullptr, *d_col = nullptr, *d_eid = nullptr, *d_dst = nullptr;
+
+    // Allocation bookkeeping.
+    bool has_alloc = false;
+    ug_allocator alloc{};
+    std::vector<void *> owned;
+    int device = 0;
+
+    // Table 7 statistics.
+    double mean_deg = 0.0, std_nnz = 0.0;
+    int64_t max_deg = 0;
+
+    // UG_SV plans keyed by chunk size.
+    mutable std::mutex mu;
+    mutable std::map<int, ug::SplitPlan> plans;
+    mutable std::vector<void *> plan_allocs;
+};

@@ -1,0 +1,412 @@
+// ug_op.cpp -- the unified operator entry point (uGrapher(Graph_Tensor, op_info,
+// parallel_info)): validation against the op set (Table 4,
+// PAPER.md:291-307; Table 2), lowering (the paper's two code-generation
+// passes, done as template selection), schedule resolution and launch.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+
+#include "ug_internal.h"
+#include "ug_runtime.h"
+
+namespace ug {
+
+static thread_local std::string g_last_error;
+
+ug_status set_error(ug_status s, const std::string &msg) {
+    g_last_error = msg;
+    return s;
+}
+
+static int pow2ceil(int64_t x) {
+    int p = 1;
+    while (p < x && p < (1 << 30)) p <<= 1;
+    return p;
+}
+
+static bool is_pow2(int x) { return x > 0 && (x & (x - 1)) == 0; }
+
+// ------------------------------------------------------------------------- lowering
+ug_status lower(const ug_graph *g, const ug_op_info *op, Lowered *out) {
+    if (!g || !op || !out) return set_error(UG_ERR_INVALID_ARG, "NULL graph / op_info");
+    const int eo = op->edge_op, go = op->gather_op;
+    if (eo < UG_EDGE_COPY_LHS || eo > UG_EDGE_DOT) return set_error(UG_ERR_INVALID_ARG, "edge_op out of range");
+    if (go < UG_GATHER_ASSIGN || go > UG_GATHER_MEAN) return set_error(UG_ERR_INVALID_ARG, "gather_op out of range");
+    const int F = op->feat, H = op->heads;
+    if (F <= 0 || H <= 0 || F % H != 0) return set_error(UG_ERR_SHAPE, "need F > 0, H > 0 and H | F");
+    const ug_tensor &C = op->C;
+    if (C.type != UG_T_DST_V && C.type != UG_T_EDGE)
+        return set_error(UG_ERR_UNSUPPORTED_OP, "C must be a Dst_V (aggregation) or Edge (message creation) tensor");
+    const bool to_edges = C.type == UG_T_EDGE;
+    if (to_edges != (go == UG_GATHER_ASSIGN))
+        return set_error(UG_ERR_UNSUPPORTED_OP,
+                         "gather assign writes edges; sum/max/min/mean reduce into Dst_V (Table 4)");
+    const bool dot = eo == UG_EDGE_DOT;
+    const int W = dot ? H : F;
+    if (C.width != W) return set_error(UG_ERR_SHAPE, "C width must be F (or H for dot)");
+    if (C.ld < C.width || !C.data) return set_error(UG_ERR_SHAPE, "C: ld < width or NULL data");
+
+    // Pass 1: copy ops use one operand; copy_rhs is copy_lhs on B.
+    const ug_tensor *opa = nullptr, *opb = nullptr;
+    if (eo == UG_EDGE_COPY_LHS) opa = &op->A;
+    else if (eo == UG_EDGE_COPY_RHS) opa = &op->B;
+    else { opa = &op->A; opb = &op->B; }
+    Operand oa{nullptr, UG_T_NULL, 1, 0}, ob{nullptr, UG_T_NULL, 1, 0};
+    const ug_tensor *used[2] = {opa, opb};
+    Operand *dst_ops[2] = {&oa, &ob};
+    for (int i = 0; i < 2; ++i) {
+        const ug_tensor *t = used[i];
+        if (!t) continue;
+        if (t->type != UG_T_SRC_V && t->type != UG_T_DST_V && t->type != UG_T_EDGE)
+            return set_error(UG_ERR_UNSUPPORTED_OP, "an operand the edge_op reads has type NULL");
+        if (!t->data) return set_error(UG_ERR_INVALID_ARG, "operand data is NULL");
+        if (!(t->width == F || t->width == H || t->width == 1))
+            return set_error(UG_ERR_SHAPE, "operand width must be F, H or 1");
+        if (t->ld < t->width) return set_error(UG_ERR_SHAPE, "operand ld < width");
+        dst_ops[i]->p = (const float *)t->data;
+        dst_ops[i]->type = t->type;
+        dst_ops[i]->div = F / t->width;
+        dst_ops[i]->ld = t->ld;
+    }
+    if (!opb) ob = oa;   // unused; keep valid pointers for the address arithmetic
+
+    Lowered lw{};
+    lw.dot = dot;
+    lw.gather = go;
+    lw.to_edges = to_edges;
+    lw.kedge = dot ? -1
+             : (eo <= UG_EDGE_COPY_RHS ? K_COPY
+                : eo == UG_EDGE_ADD ? K_ADD : eo == UG_EDGE_SUB ? K_SUB : eo == UG_EDGE_MUL ? K_MUL : K_DIV);
+    lw.args.A = oa;
+    lw.args.B = ob;
+    lw.args.C = (float *)C.data;
+    lw.args.c_ld = C.ld;
+    lw.args.c_type = C.type;
+    lw.args.F = F;
+    lw.args.W = W;
+    lw.args.H = H;
+    lw.args.D = F / H;
+    lw.op_class = dot ? (to_edges ? 2 : 3) : (to_edges ? 0 : 1);
+
+    // Widest legal feature vector (R22 in DESIGN.md): every full-width operand row must be
+    // aligned and either F % vec == 0 or padded (ld >= round_up(F, vec)); a broadcast operand
+    // must keep a vec chunk inside one head; C stores must be aligned.
+    lw.max_vec = 1;
+    for (int v : {4, 2}) {
+        bool ok = true;
+        const int span = dot ? lw.args.D : F;
+        for (int i = 0; i < 2 && ok; ++i) {
+            const ug_tensor *t = used[i];
+            if (!t) continue;
+            const Operand &o = *dst_ops[i];
+            if (o.div == 1) {
+                ok = (o.ld % v == 0) && ((uintptr_t)o.p % (4 * v) == 0) &&
+                     (span % v == 0 || o.ld >= ((F + v - 1) / v) * v);
+            } else {
+                ok = (o.div % v == 0);
+            }
+        }
+        if (ok && !dot) ok = (C.ld % v == 0) && ((uintptr_t)C.data % (4 * v) == 0);
+        if (ok && dot) ok = (lw.args.D % v == 0);
+        if (ok) { lw.max_vec = v; break; }
+    }
+    *out = lw;
+    return UG_OK;
+}
+
+// ------------------------------------------------------------------------- resolution
+ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, LaunchCfg *cfg) {
+    (void)g;
+    LaunchCfg c{};
+    c.strategy = s.strategy;
+    if (c.strategy < UG_TV || c.strategy > UG_SV)
+        return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "strategy out of range");
+    c.vec = s.vec ? s.vec : lw.max_vec;
+    if (!(c.vec == 1 || c.vec == 2 || c.vec == 4)) return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "vec must be 1, 2 or 4");
+    if (c.vec > lw.max_vec) return set_error(UG_ERR_ALIGNMENT, "forced vec wider than the operand layout allows");
+    c.G = s.group > 0 ? s.group : (c.strategy == UG_SV ? 2048 : 1);
+    const int T = s.tile > 0 ? s.tile : 1;
+    if (!is_pow2(T)) return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "tile T must be a power of two");
+    c.block = s.block_threads > 0 ? s.block_threads : 256;
+    const int max_block = (c.strategy == UG_BV) ? 1024 : 256;
+    if (c.block % 32 || c.block > max_block)
+        return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "block_threads must be a multiple of 32 and <= 256 (1024 for BV)");
+    // Lanes: lanes beyond the feature chunks of one unit would have no work; they are not
+    // launched (clamp rule).
+    const int span = lw.dot ? lw.args.D : lw.args.W;
+    const int need = pow2ceil((span + c.vec - 1) / c.vec);
+    switch (c.strategy) {
+    case UG_TV: case UG_TE: c.L = T; break;
+    case UG_WV: case UG_WE: c.L = 32 * T; break;
+    default: c.L = 32; break;
+    }
+    c.L = std::max(1, std::min(c.L, need));
+    if (lw.dot) c.L = std::min(c.L, 32);
+    c.ftile = s.ftile;
+    if (c.ftile < 0 || c.ftile % c.vec) return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "ftile must be a multiple of vec");
+    if (c.strategy == UG_SV && !lw.dot) {
+        if (c.ftile == 0) c.ftile = std::min(32, need) * c.vec;
+        const int L = c.ftile / c.vec;
+        if (!is_pow2(L) || L > 32)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "SV needs ftile / vec a power of two <= 32");
+        c.L = L;
+    }
+    if (c.strategy == UG_BE) c.L = std::min(32, need);
+    *cfg = c;
+    return UG_OK;
+}
+
+static GraphArgs graph_args(const ug_graph *g) {
+    GraphArgs a;
+    a.row_ptr = g->d_row_ptr;
+    a.col = g->d_col;
+    a.eid = g->d_eid;
+    a.dst = g->d_dst;
+    a.V = g->V;
+    a.E = g->E;
+    a.rp_base = g->e0;
+    a.r0 = g->r0;
+    return a;
+}
+
+// Split-row plan for UG_SV (cached per chunk size; uploaded synchronously on first use).
+static ug_status get_plan(const ug_graph *g, int G, const SplitPlan **out) {
+    std::lock_guard<std::mutex> lock(g->mu);
+    auto it = g->plans.find(G);
+    if (it != g->plans.end()) { *out = &it->second; return UG_OK; }
+    std::vector<int32_t> chunks, split;
+    int64_t slot = 0;
+    for (int64_t v = 0; v < g->V; ++v) {
+        const int64_t k0 = (int64_t)g->h_row_ptr[v] - g->e0, k1 = (int64_t)g->h_row_ptr[v + 1] - g->e0;
+        const int64_t n = std::max<int64_t>(1, (k1 - k0 + G - 1) / G);
+        if (n == 1) {
+            chunks.insert(chunks.end(), {(int32_t)v, (int32_t)k0, (int32_t)k1, -1});
+        } else {
+            split.insert(split.end(), {(int32_t)v, (int32_t)slot, (int32_t)n, 0});
+            for (int64_t i = 0; i < n; ++i) {
+                const int64_t a = k0 + i * G, b = std::min(k1, a + G);
+                chunks.insert(chunks.end(), {(int32_t)v, (int32_t)a, (int32_t)b, (int32_t)slot++});
+            }
+        }
+    }
+    SplitPlan p;
+    p.n_chunks = (int64_t)chunks.size() / 4;
+    p.n_split_rows = (int64_t)split.size() / 4;
+    p.n_split_chunks = slot;
+    void *dc = nullptr, *ds = nullptr;
+    if (cudaMalloc(&dc, std::max<size_t>(16, chunks.size() * 4)) != cudaSuccess ||
+        cudaMalloc(&ds, std::max<size_t>(16, split.size() * 4)) != cudaSuccess)
+        return set_error(UG_ERR_OOM, "SV plan allocation failed");
+    g->plan_allocs.push_back(dc);
+    g->plan_allocs.push_back(ds);
+    if ((!chunks.empty() && cudaMemcpy(dc, chunks.data(), chunks.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) ||
+        (!split.empty() && cudaMemcpy(ds, split.data(), split.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess))
+        return set_error(UG_ERR_CUDA, "SV plan upload failed");
+    p.d_chunk = (int32_t *)dc;
+    p.d_split = (int32_t *)ds;
+    auto res = g->plans.emplace(G, p);
+    *out = &res.first->second;
+    return UG_OK;
+}
+
+static int launches_for(const Lowered &lw, const LaunchCfg &c, int64_t n_split_rows) {
+    const bool edge_units = c.strategy == UG_TE || c.strategy == UG_WE || c.strategy == UG_BE;
+    if (lw.to_edges) return 1;
+    if (edge_units) return lw.gather == UG_GATHER_SUM ? 2 : 3;
+    if (c.strategy == UG_SV && !lw.dot) return n_split_rows > 0 ? 2 : 1;
+    return 1;
+}
+
+static void ensure_pool_retains() {
+    static bool done = false;
+    if (done) return;
+    done = true;
+    int dev = 0;
+    cudaMemPool_t pool;
+    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+}
+
+}  // namespace ug
+
+using namespace ug;
+
+extern "C" ug_status ug_op_validate(const ug_graph *g, const ug_op_info *op) {
+    Lowered lw;
+    return lower(g, op, &lw);
+}
+
+static ug_status prepare(const ug_graph *g, const ug_op_info *op, const ug_schedule *sched, Lowered *lw,
+                         LaunchCfg *cfg) {
+    ug_status st = lower(g, op, lw);
+    if (st != UG_OK) return st;
+    ug_schedule s{};
+    if (sched && sched->strategy != UG_SCHED_AUTO) s = *sched;
+    else if ((st = select_schedule(g, *lw, &s)) != UG_OK) return st;
+    return resolve(g, *lw, s, cfg);
+}
+
+extern "C" ug_status ug_op_launch_count(const ug_graph *g, const ug_op_info *op, const ug_schedule *sched,
+                                        int32_t *launches) {
+    Lowered lw;
+    LaunchCfg c;
+    if (!launches) return set_error(UG_ERR_INVALID_ARG, "NULL out");
+    ug_status st = prepare(g, op, sched, &lw, &c);
+    if (st != UG_OK) return st;
+    int64_t nsr = 0;
+    if (c.strategy == UG_SV && !lw.dot && !lw.to_edges) {
+        // count split rows on the host without touching the device
+        for (int64_t v = 0; v < g->V; ++v)
+            if ((int64_t)g->h_row_ptr[v + 1] - g->h_row_ptr[v] > c.G) ++nsr;
+    }
+    *launches = launches_for(lw, c, nsr);
+    return UG_OK;
+}
+
+static ug_status run(const ug_graph *g, const ug_op_info *op, const ug_schedule *sched, void *stream,
+                     cudaEvent_t ev_begin, cudaEvent_t ev_end) {
+    Lowered lw;
+    LaunchCfg c;
+    ug_status st = prepare(g, op, sched, &lw, &c);
+    if (st != UG_OK) return st;
+    if (g->host_only) return set_error(UG_ERR_INVALID_ARG, "ug_op_run needs a device graph (not UG_GRAPH_HOST_ONLY)");
+    cudaStream_t s = (cudaStream_t)stream;
+    const GraphArgs ga = graph_args(g);
+    const bool edge_units = c.strategy == UG_TE || c.strategy == UG_WE || c.strategy == UG_BE;
+    cudaError_t err = cudaSuccess;
+    const bool agg = !lw.to_edges;
+    if (edge_units && agg) {
+        err = launch_init(lw.gather, lw.args, g->V, s);
+        if (err == cudaSuccess) {
+            LaunchCfg ce = c;
+            if (c.strategy == UG_BE) ce.L = std::min(c.L, 32);
+            if (ev_begin) cudaEventRecord(ev_begin, s);
+            err = lw.dot ? launch_dot(false, lw.gather, ga, lw.args, ce, s)
+                         : launch_edge(lw.kedge, lw.gather, ga, lw.args, ce, s);
+            if (ev_end) cudaEventRecord(ev_end, s);
+        }
+        if (err == cudaSuccess && lw.gather != UG_GATHER_SUM) err = launch_epilogue(lw.gather, ga, lw.args, s);
+    } else if (lw.dot) {
+        if (ev_begin) cudaEventRecord(ev_begin, s);
+        err = launch_dot(!edge_units, lw.gather, ga, lw.args, c, s);
+        if (ev_end) cudaEventRecord(ev_end, s);
+    } else if (edge_units) {
+        if (ev_begin) cudaEventRecord(ev_begin, s);
+        err = launch_edge(lw.kedge, lw.gather, ga, lw.args, c, s);
+        if (ev_end) cudaEventRecord(ev_end, s);
+    } else if (c.strategy == UG_TV || c.strategy == UG_WV) {
+        if (ev_begin) cudaEventRecord(ev_begin, s);
+        err = launch_vertex(lw.kedge, lw.gather, ga, lw.args, c, s);
+        if (ev_end) cudaEventRecord(ev_end, s);
+    } else if (c.strategy == UG_BV) {
+        if (ev_begin) cudaEventRecord(ev_begin, s);
+        err = launch_block_vertex(lw.kedge, lw.gather, ga, lw.args, c, s);
+        if (ev_end) cudaEventRecord(ev_end, s);
+    } else {  // UG_SV
+        const SplitPlan *plan = nullptr;
+        if ((st = get_plan(g, c.G, &plan)) != UG_OK) return st;
+        float *scratch = nullptr;
+        const int64_t sld = (lw.args.W + 3) / 4 * 4;
+        if (agg && plan->n_split_chunks > 0) {
+            ensure_pool_retains();
+            err = cudaMallocAsync((void **)&scratch, sizeof(float) * (size_t)(plan->n_split_chunks * sld), s);
+            if (err != cudaSuccess) return set_error(UG_ERR_OOM, "SV scratch allocation failed");
+        }
+        err = launch_split_vertex(lw.kedge, lw.gather, ga, lw.args, c, *plan, scratch, s, ev_begin, ev_end);
+        if (scratch) cudaFreeAsync(scratch, s);
+    }
+    if (err != cudaSuccess) return set_error(UG_ERR_CUDA, std::string("kernel launch: ") + cudaGetErrorString(err));
+    return UG_OK;
+}
+
+extern "C" ug_status ug_op_run(const ug_graph *g, const ug_op_info *op, const ug_schedule *sched, void *stream) {
+    return run(g, op, sched, stream, nullptr, nullptr);
+}
+
+extern "C" ug_status ug_op_run_events(const ug_graph *g, const ug_op_info *op, const ug_schedule *sched,
+                                      void *stream, void *ev_begin, void *ev_end) {
+    return run(g, op, sched, stream, (cudaEvent_t)ev_begin, (cudaEvent_t)ev_end);
+}
+
+extern "C" ug_status ug_edge_permute(const ug_graph *g, const float *in, float *out, int32_t width, void *stream) {
+    if (!g || !in || !out || width <= 0) return set_error(UG_ERR_INVALID_ARG, "ug_edge_permute: bad arguments");
+    if (g->host_only) return set_error(UG_ERR_INVALID_ARG, "ug_edge_permute needs a device graph");
+    cudaError_t e = launch_permute(g->d_eid, in, out, g->E, width, (cudaStream_t)stream);
+    if (e != cudaSuccess) return set_error(UG_ERR_CUDA, cudaGetErrorString(e));
+    return UG_OK;
+}
+
+// ------------------------------------------------------------------------- text form
+static const char *kStrat[] = {"AUTO", "TV", "TE", "WV", "WE", "BV", "BE", "SV"};
+
+extern "C" ug_status ug_schedule_parse(const char *text, ug_schedule *out) {
+    if (!text || !out) return set_error(UG_ERR_INVALID_ARG, "ug_schedule_parse: NULL");
+    ug_schedule s{};
+    std::string t(text);
+    size_t pos = t.find('_');
+    std::string head = t.substr(0, pos);
+    int strat = -1;
+    for (int i = 0; i < 8; ++i)
+        if (head == kStrat[i]) strat = i;
+    if (strat < 0) return set_error(UG_ERR_INVALID_ARG, "unknown strategy '" + head + "'");
+    s.strategy = strat;
+    while (pos != std::string::npos) {
+        size_t nxt = t.find('_', pos + 1);
+        std::string tok = t.substr(pos + 1, nxt == std::string::npos ? std::string::npos : nxt - pos - 1);
+        if (tok.size() < 2) return set_error(UG_ERR_INVALID_ARG, "bad schedule token '" + tok + "'");
+        char *end = nullptr;
+        long val = std::strtol(tok.c_str() + 1, &end, 10);
+        if (*end != '\0' || val < 0) return set_error(UG_ERR_INVALID_ARG, "bad schedule token '" + tok + "'");
+        switch (tok[0]) {
+        case 'G': s.group = (int32_t)val; break;
+        case 'T': s.tile = (int32_t)val; break;
+        case 'B': s.block_threads = (int32_t)val; break;
+        case 'F': s.ftile = (int32_t)val; break;
+        case 'V': s.vec = (int32_t)val; break;
+        default: return set_error(UG_ERR_INVALID_ARG, "bad schedule token '" + tok + "'");
+        }
+        pos = nxt;
+    }
+    *out = s;
+    return UG_OK;
+}
+
+extern "C" ug_status ug_schedule_format(const ug_schedule *s, char *buf, size_t len) {
+    if (!s || !buf || s->strategy < 0 || s->strategy > 7) return set_error(UG_ERR_INVALID_ARG, "ug_schedule_format: bad args");
+    std::string r = kStrat[s->strategy];
+    if (s->strategy != UG_SCHED_AUTO) {
+        r += "_G" + std::to_string(s->group > 0 ? s->group : (s->strategy == UG_SV ? 2048 : 1));
+        if (s->strategy != UG_SV && s->strategy != UG_BV && s->strategy != UG_BE)
+            r += "_T" + std::to_string(s->tile > 0 ? s->tile : 1);
+        if (s->ftile) r += "_F" + std::to_string(s->ftile);
+        if (s->block_threads) r += "_B" + std::to_string(s->block_threads);
+        if (s->vec) r += "_V" + std::to_string(s->vec);
+    }
+    std::snprintf(buf, len, "%s", r.c_str());
+    return UG_OK;
+}
+
+extern "C" const char *ug_status_string(ug_status s) {
+    switch (s) {
+    case UG_OK: return "UG_OK";
+    case UG_ERR_INVALID_ARG: return "UG_ERR_INVALID_ARG";
+    case UG_ERR_UNSUPPORTED_OP: return "UG_ERR_UNSUPPORTED_OP";
+    case UG_ERR_SHAPE: return "UG_ERR_SHAPE";
+    case UG_ERR_INDEX_RANGE: return "UG_ERR_INDEX_RANGE";
+    case UG_ERR_ALIGNMENT: return "UG_ERR_ALIGNMENT";
+    case UG_ERR_OOM: return "UG_ERR_OOM";
+    case UG_ERR_CUDA: return "UG_ERR_CUDA";
+    case UG_ERR_UNSUPPORTED_SCHEDULE: return "UG_ERR_UNSUPPORTED_SCHEDULE";
+    }
+    return "UG_ERR_UNKNOWN";
+}
+
+extern "C" const char *ug_last_error(void) { return g_last_error.c_str(); }
+
+extern "C" const char *ug_version(void) { return "ugraph-b200 0.1 (sm_100a)"; }

@@ -1,0 +1,33 @@
+// ug_runtime.h -- host-side helpers shared by the runtime translation units.
+#pragma once
+#include <string>
+
+#include "ug.h"
+#include "ug_internal.h"
+
+namespace ug {
+
+ug_status set_error(ug_status s, const std::string &msg);
+
+// Operator after lowering (validation + pass 1 of PAPER.md:405: copy ops fused, copy_rhs
+// rewritten as copy_lhs on B, operand broadcast factors resolved).
+struct Lowered {
+    int kedge;          // K_COPY .. K_DIV, or -1 for dot
+    bool dot;
+    int gather;         // UG_GATHER_*
+    bool to_edges;      // C is an Edge tensor (message creation)
+    OpArgs args;
+    int max_vec;        // widest legal feature vector (1, 2, 4)
+    // selector key
+    int op_class;       // 0 msg, 1 agg, 2 dot msg, 3 dot agg
+};
+
+ug_status lower(const ug_graph *g, const ug_op_info *op, Lowered *out);
+
+// Concrete launch configuration for a (graph, lowered op, schedule).
+ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, LaunchCfg *cfg);
+
+// Selector (ug_selector.cpp).
+ug_status select_schedule(const ug_graph *g, const Lowered &lw, ug_schedule *out);
+
+}  // namespace ug

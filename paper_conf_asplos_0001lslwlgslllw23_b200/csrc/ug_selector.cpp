@@ -1,0 +1,188 @@
+// ug_selector.cpp -- schedule selection when parallel_info is absent.
+//
+// The paper trains LightGBM on Table 7's features; this build replaces the
+// learned model by a table of schedules MEASURED on B200 (bench/sweep.py writes
+// selector_table.json), keyed by the Table 7 features plus the feature width F that Fig. 7
+// shows matters: op class, F, mean in-degree, degree CV (= std_nnz /
+// mean), V.  First matching entry wins; no match falls back to the priors below (Table 9's
+// observations, re-derived for B200 in DESIGN.md).  Lookup is a linear scan
+// over a few hundred entries: well under the paper's 0.2 ms budget.
+#include <dlfcn.h>
+
+#include <cctype>
+#include <cstdlib>
+#include <cstring>
+#include <fstream>
+#include <mutex>
+#include <sstream>
+#include <string>
+#include <vector>
+
+#include "ug_internal.h"
+#include "ug_runtime.h"
+
+namespace ug {
+
+struct Entry {
+    int op_class = -1;          // -1 = any
+    double F_lo = 0, F_hi = 1e18, deg_lo = 0, deg_hi = 1e18, cv_lo = 0, cv_hi = 1e18, V_lo = 0, V_hi = 1e18;
+    ug_schedule sched{};
+};
+
+static std::mutex g_mu;
+static std::vector<Entry> g_table;
+static bool g_loaded = false;
+
+static int class_of(const std::string &s) {
+    if (s == "msg") return 0;
+    if (s == "agg") return 1;
+    if (s == "dot_msg") return 2;
+    if (s == "dot_agg") return 3;
+    return -1;
+}
+
+// Minimal JSON reader for {"entries": [{"key": number | "string", ...}, ...]}.
+static bool parse_table(const std::string &txt, std::vector<Entry> *out, std::string *why) {
+    size_t p = txt.find("\"entries\"");
+    if (p == std::string::npos) { *why = "no \"entries\" key"; return false; }
+    p = txt.find('[', p);
+    if (p == std::string::npos) { *why = "entries is not an array"; return false; }
+    std::vector<Entry> res;
+    while (true) {
+        size_t ob = txt.find_first_of("{]", p + 1);
+        if (ob == std::string::npos) { *why = "unterminated entries"; return false; }
+        if (txt[ob] == ']') break;
+        size_t cb = txt.find('}', ob);
+        if (cb == std::string::npos) { *why = "unterminated object"; return false; }
+        std::string obj = txt.substr(ob + 1, cb - ob - 1);
+        Entry e;
+        size_t q = 0;
+        while ((q = obj.find('"', q)) != std::string::npos) {
+            size_t qe = obj.find('"', q + 1);
+            if (qe == std::string::npos) break;
+            std::string key = obj.substr(q + 1, qe - q - 1);
+            size_t colon = obj.find(':', qe);
+            if (colon == std::string::npos) break;
+            size_t vs = colon + 1;
+            while (vs < obj.size() && std::isspace((unsigned char)obj[vs])) ++vs;
+            std::string sval;
+            double nval = 0;
+            bool is_str = vs < obj.size() && obj[vs] == '"';
+            size_t ve;
+            if (is_str) {
+                ve = obj.find('"', vs + 1);
+                sval = obj.substr(vs + 1, ve - vs - 1);
+                ++ve;
+            } else {
+                ve = obj.find_first_of(",}", vs);
+                if (ve == std::string::npos) ve = obj.size();
+                nval = std::strtod(obj.substr(vs, ve - vs).c_str(), nullptr);
+            }
+            if (key == "class") e.op_class = class_of(sval);
+            else if (key == "F_lo") e.F_lo = nval;
+            else if (key == "F_hi") e.F_hi = nval;
+            else if (key == "deg_lo") e.deg_lo = nval;
+            else if (key == "deg_hi") e.deg_hi = nval;
+            else if (key == "cv_lo") e.cv_lo = nval;
+            else if (key == "cv_hi") e.cv_hi = nval;
+            else if (key == "V_lo") e.V_lo = nval;
+            else if (key == "V_hi") e.V_hi = nval;
+            else if (key == "schedule") {
+                if (ug_schedule_parse(sval.c_str(), &e.sched) != UG_OK) { *why = "bad schedule " + sval; return false; }
+            }
+            q = ve;
+        }
+        if (e.sched.strategy != UG_SCHED_AUTO) res.push_back(e);
+        p = cb;
+    }
+    *out = std::move(res);
+    return true;
+}
+
+static std::string default_table_path() {
+    const char *env = std::getenv("UG_SELECTOR_TABLE");
+    if (env && *env) return env;
+    Dl_info info;
+    if (dladdr((void *)&default_table_path, &info) && info.dli_fname) {
+        std::string f(info.dli_fname);
+        size_t sl = f.rfind('/');
+        return (sl == std::string::npos ? std::string(".") : f.substr(0, sl)) + "/selector_table.json";
+    }
+    return "selector_table.json";
+}
+
+static ug_status load_file(const std::string &path, bool quiet) {
+    std::ifstream in(path);
+    if (!in) return quiet ? UG_OK : set_error(UG_ERR_INVALID_ARG, "cannot open " + path);
+    std::stringstream ss;
+    ss << in.rdbuf();
+    std::vector<Entry> t;
+    std::string why;
+    if (!parse_table(ss.str(), &t, &why)) return set_error(UG_ERR_INVALID_ARG, "selector table " + path + ": " + why);
+    g_table = std::move(t);
+    return UG_OK;
+}
+
+// Priors used when no measured entry matches.
+static ug_schedule prior(const ug_graph *g, const Lowered &lw) {
+    ug_schedule s{};
+    const int W = lw.args.W, vec = lw.max_vec;
+    const int chunks = (W + vec - 1) / vec;
+    int lanes = 1;
+    while (lanes < chunks && lanes < 32) lanes <<= 1;
+    if (lw.op_class == 0) {            // message creation: thread-edge (Table 9: always TE)
+        s.strategy = UG_TE; s.group = 1; s.tile = lanes;
+    } else if (lw.op_class == 2) {     // SDDMM: lanes over the head's D features
+        int dl = 1;
+        const int dch = (lw.args.D + vec - 1) / vec;
+        while (dl < dch && dl < 32) dl <<= 1;
+        s.strategy = UG_TE; s.group = 1; s.tile = dl;
+    } else if (lw.op_class == 3) {
+        s.strategy = UG_WV; s.group = 1; s.tile = 1;
+    } else {                           // aggregation
+        if (W >= 32 || g->max_deg > 256) { s.strategy = UG_SV; s.group = 1024; s.ftile = 0; }
+        else { s.strategy = UG_WV; s.group = 1; s.tile = 1; }
+    }
+    return s;
+}
+
+ug_status select_schedule(const ug_graph *g, const Lowered &lw, ug_schedule *out) {
+    const char *force = std::getenv("UG_FORCE_SCHEDULE");
+    if (force && *force) return ug_schedule_parse(force, out);
+    std::lock_guard<std::mutex> lock(g_mu);
+    if (!g_loaded) {
+        g_loaded = true;
+        load_file(default_table_path(), true);
+    }
+    const double F = lw.args.F, deg = g->mean_deg, V = (double)g->V;
+    const double cv = g->mean_deg > 0 ? g->std_nnz / g->mean_deg : 0.0;
+    for (const Entry &e : g_table) {
+        if (e.op_class != -1 && e.op_class != lw.op_class) continue;
+        if (F < e.F_lo || F > e.F_hi || deg < e.deg_lo || deg > e.deg_hi || cv < e.cv_lo || cv > e.cv_hi ||
+            V < e.V_lo || V > e.V_hi)
+            continue;
+        ug_schedule s = e.sched;
+        if (s.vec > lw.max_vec) s.vec = 0;   // table entry measured on an aligned layout
+        *out = s;
+        return UG_OK;
+    }
+    *out = prior(g, lw);
+    return UG_OK;
+}
+
+}  // namespace ug
+
+extern "C" ug_status ug_schedule_select(const ug_graph *g, const ug_op_info *op, ug_schedule *out) {
+    if (!out) return ug::set_error(UG_ERR_INVALID_ARG, "NULL out");
+    ug::Lowered lw;
+    ug_status st = ug::lower(g, op, &lw);
+    if (st != UG_OK) return st;
+    return ug::select_schedule(g, lw, out);
+}
+
+extern "C" ug_status ug_selector_load(const char *path) {
+    if (!path) return ug::set_error(UG_ERR_INVALID_ARG, "NULL path");
+    std::lock_guard<std::mutex> lock(ug::g_mu);
+    ug::g_loaded = true;
+    return ug::load_file(path, false);
+}

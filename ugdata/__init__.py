@@ -30,20 +30,21 @@ class GraphConfig:
     seed: int
     widths: tuple      # feature widths F exercised by this config
     note: str
+    label: str = ""
 
 
 # BASELINE.json configs; shapes and skew per SURVEY.md 8(d) (Table 3).
 CONFIGS = {
     "C1": GraphConfig("C1", 2708, 10556, False, 1.015, 1.015, 1001, (16,),
-                      "Cora-shaped (PAPER.md:148): u_mul_e_sum F=16"),
+                      "Cora-shaped (PAPER.md:148): u_mul_e_sum F=16", "Cora-shaped"),
     "C2": GraphConfig("C2", 19717, 88648, False, 1.108, 1.108, 1002, (16, 64),
-                      "Pubmed-shaped (PAPER.md:150, E per BASELINE.json): GAT op set"),
+                      "Pubmed-shaped (PAPER.md:150, E per BASELINE.json): GAT op set", "Pubmed-shaped"),
     "C3": GraphConfig("C3", 403394, 3387388, True, 1.209, 0.5, 1003, (32, 64, 128),
-                      "amazon0601-shaped (PAPER.md:157): GCN/GIN aggregation, schedule sweep"),
+                      "amazon0601-shaped (PAPER.md:157): GCN/GIN aggregation, schedule sweep", "amazon0601-shaped"),
     "C4": GraphConfig("C4", 169343, 1166243, True, 1.2, 0.5, 1004, (128, 256),
-                      "ogbn-arxiv-shaped: u_dot_v SDDMM"),
+                      "ogbn-arxiv-shaped: u_dot_v SDDMM", "ogbn-arxiv-shaped"),
     "C5": GraphConfig("C5", 232965, 114615892, False, 1.0, 1.0, 1005, (602,),
-                      "Reddit-shaped: copy_u_sum / copy_u_mean F=602"),
+                      "Reddit-shaped: copy_u_sum / copy_u_mean F=602", "Reddit-shaped"),
 }
 
 
