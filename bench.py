@@ -176,46 +176,39 @@ def main():
 
     import torch
     import paper_conf_asplos_0001lslwlgslllw23_b200 as ug
+    from paper_conf_asplos_0001lslwlgslllw23_b200.pipeline import StreamedOperator
+    from paper_conf_asplos_0001lslwlgslllw23_b200.shard import ShardedOperator, x_block
 
     dist = None
     if world > 1:
         import torch.distributed as dist
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local if world > 1 else 0)
+    dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
 
     src, dst = ugdata.graph(args.config)
     V, E = cfg.V, len(src)
     eo, go, a_t, b_t = OPS[args.op]
     g_full = ug.Graph(V, src, dst)
+    sh = ShardedOperator(g_full, world, rank)
+    g = sh.view
+    Vl, El = sh.local_rows, sh.e1 - sh.e0
 
-    # shard: edge-balanced destination rows (R21); X row blocks of ceil(V/P) for the all-gather
-    if world > 1:
-        splits = g_full.partition(world)
-        r0, r1 = int(splits[rank]), int(splits[rank + 1])
-        g = g_full.view_rows(r0, r1)
-    else:
-        r0, r1 = 0, V
-        g = g_full
-    Vl = r1 - r0
-    blk = -(-V // world)
     X_host = ugdata.values(V, F, cfg.seed + 1, 1)
-    X_full = torch.empty(blk * world, F, device=dev)
+    X_full = torch.empty(sh.blk * world, F, device=dev)
     X_full[:V].copy_(torch.from_numpy(X_host))
-    X_local = X_full[rank * blk:(rank + 1) * blk].clone() if world > 1 else None
+    X_local = x_block(X_full[:V], V, world, rank)
     Bt = None
     if b_t == "e":
-        rp = g_full.csr()[0] if world > 1 else None
-        wE = torch.from_numpy(ugdata.values(E, 1, cfg.seed + 1, 2, role="edge")).to(dev)
-        Bt = wE[int(rp[r0]):int(rp[r1])] if world > 1 else wE
+        Bt = sh.edge_slice(torch.from_numpy(ugdata.values(E, 1, cfg.seed + 1, 2, role="edge")).to(dev))
     elif b_t == "v":
-        Bt = X_full[r0:r1]
-    Y = torch.empty(Vl if go != "assign" else g.stats()["E"], F if eo != "dot" else 1, device=dev)
-    sched = args.schedule
-    kw = dict(A=X_full[:V], a_type=a_t, B=Bt, b_type=b_t, C=Y, c_type="e" if go == "assign" else "v",
-              F=F, H=1)
-    chosen = sched or ug.schedule_select(g, eo, go, **kw)
+        Bt = sh.dst_slice(X_full)
+    c_t = "e" if go == "assign" else "v"
+    W = 1 if eo == "dot" else F
+    Y = torch.empty(Vl if c_t == "v" else El, W, device=dev)
+    kw = dict(A=X_full[:V], a_type=a_t, B=Bt, b_type=b_t, C=Y, c_type=c_t, F=F, H=1)
+    chosen = args.schedule or ug.schedule_select(g, eo, go, **kw)
     launches = ug.launch_count(g, eo, go, schedule=chosen, **kw)
 
     stream = torch.cuda.current_stream(dev)
@@ -229,7 +222,7 @@ def main():
 
     def step(i=None):
         if world > 1:
-            dist.all_gather_into_tensor(X_full, X_local)
+            sh.gather_x(X_local, X_full)          # the exchange: NCCL all-gather of X row blocks
         if i is None:
             ug.op_run(g, eo, go, schedule=chosen, **kw)
         else:
@@ -250,10 +243,8 @@ def main():
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    step_ms = [ev_s0[i].elapsed_time(ev_s1[i]) for i in range(args.steps)]
-    kern_ms = [ev_k0[i].elapsed_time(ev_k1[i]) for i in range(args.steps)]
-    tot = sum(step_ms)
-    ktot = sum(kern_ms)
+    tot = sum(ev_s0[i].elapsed_time(ev_s1[i]) for i in range(args.steps))
+    ktot = sum(ev_k0[i].elapsed_time(ev_k1[i]) for i in range(args.steps))
     if world > 1:
         t = torch.tensor([tot, ktot], device=dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -261,47 +252,62 @@ def main():
     ms = tot / args.steps
     kms = ktot / args.steps
     by = logical_bytes(V, E, F, args.op)
-    by_local = logical_bytes(Vl, g.stats()["E"], F, args.op)
+    by_local = logical_bytes(Vl, El, F, args.op)
     value = by / (ms * 1e-3) / 1e9
     peak, peak_src = load_peaks()
     achieved = by_local / (kms * 1e-3) / 1e9
 
-    # e2e through the public API: pinned host X -> device, op, device Y -> pinned host.
+    # e2e through the public API (StreamedOperator): every step copies its X from pinned host
+    # memory and reads its Y back; copies of neighbouring steps overlap the operator.
     e2e = None
-    if not args.no_e2e and world == 1:
+    if not args.no_e2e:
         Xh = torch.from_numpy(X_host).pin_memory()
-        Yh = torch.empty(Y.shape, dtype=torch.float32).pin_memory()
-        Xd = torch.empty(V, F, device=dev)
-        kwe = dict(kw)
-        kwe["A"] = Xd
-        if b_t == "v":
-            kwe["B"] = Xd
-        for _ in range(2):
-            Xd.copy_(Xh, non_blocking=True)
-            ug.op_run(g, eo, go, schedule=chosen, **kwe)
-            Yh.copy_(Y, non_blocking=True)
-        torch.cuda.synchronize()
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        n_e2e = max(3, min(args.steps, 5))
-        e0.record(stream)
-        for _ in range(n_e2e):
-            Xd.copy_(Xh, non_blocking=True)
-            ug.op_run(g, eo, go, schedule=chosen, **kwe)
-            Yh.copy_(Y, non_blocking=True)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        e_ms = e0.elapsed_time(e1) / n_e2e
+        n_e2e = max(3, min(args.steps, 8))
+        Yh = [torch.empty(tuple(Y.shape), dtype=torch.float32).pin_memory() for _ in range(2)]
+        if world == 1:
+            so = StreamedOperator(g, eo, go, a_type=a_t, in_shape=(V, F), out_shape=tuple(Y.shape), c_type=c_t,
+                                  schedule=chosen, depth=2, F=F, H=1,
+                                  B=Bt if b_t == "e" else None, b_type=b_t)
+            bfn = (lambda i, Xd: Xd) if b_t == "v" else None
+            so.run([Xh] * 2, Yh, b_fn=bfn)      # warm-up
+            so.synchronize()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(so.s_in)
+            so.run([Xh] * n_e2e, [Yh[i % 2] for i in range(n_e2e)], b_fn=bfn)
+            so.s_in.wait_stream(so.s_out)
+            e1.record(so.s_in)
+            so.synchronize()
+            e_ms = e0.elapsed_time(e1) / n_e2e
+        else:
+            Xlh = torch.from_numpy(x_block(torch.from_numpy(X_host), V, world, rank).numpy()).pin_memory()
+            Xl = torch.empty_like(X_local)
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            dist.barrier()
+            e0.record(stream)
+            for i in range(n_e2e):
+                Xl.copy_(Xlh, non_blocking=True)
+                sh.gather_x(Xl, X_full)
+                ug.op_run(g, eo, go, schedule=chosen, **kw)
+                Yh[i % 2].copy_(Y, non_blocking=True)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            t = torch.tensor([e0.elapsed_time(e1) / n_e2e], device=dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e_ms = float(t[0])
         e2e = {"value": round(by / (e_ms * 1e-3) / 1e9, 1), "unit": "GB/s", "ms_per_step": round(e_ms, 3),
-               "h2d_bytes_per_step": int(Xh.numel() * 4), "d2h_bytes_per_step": int(Yh.numel() * 4)}
+               "h2d_bytes_per_step": int((V if world == 1 else sh.blk * world) * F * 4),
+               "d2h_bytes_per_step": int(Y.numel() * 4 * world),
+               "how": "pinned host X -> device, op, device Y -> pinned host, every step; copies of "
+                      "neighbouring steps overlap the op (StreamedOperator)" if world == 1 else
+                      "pinned host X block -> device, all-gather, op, Y shard -> host, every step"}
 
     traffic = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
         try:
-            tj = json.load(open(tp))
-            key = f"{args.config}:{args.op}:{F}:{chosen}"
-            traffic = tj.get(key)
+            traffic = json.load(open(tp)).get(f"{args.config}:{args.op}:{F}:{chosen}")
         except (ValueError, OSError):
             traffic = None
 
@@ -329,7 +335,7 @@ def main():
                          "frac": round(achieved / peak, 4), "traffic": traffic,
                          "kernel": "k_split (SV main traversal)" if chosen.startswith("SV") else "main traversal",
                          "kernel_ms": round(kms, 4), "peak_source": peak_src,
-                         "bytes": "algorithmic (SURVEY 8(d)) per launch"},
+                         "bytes": "algorithmic (SURVEY 8(d)) per launch, this rank's rows"},
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches * args.steps,

@@ -48,7 +48,10 @@ ug_status lower(const ug_graph *g, const ug_op_info *op, Lowered *out) {
     const bool dot = eo == UG_EDGE_DOT;
     const int W = dot ? H : F;
     if (C.width != W) return set_error(UG_ERR_SHAPE, "C width must be F (or H for dot)");
-    if (C.ld < C.width || !C.data) return set_error(UG_ERR_SHAPE, "C: ld < width or NULL data");
+    if (C.ld < C.width) return set_error(UG_ERR_SHAPE, "C: ld < width");
+    // NULL data is legal only for a tensor with zero rows (e.g. Edge tensors of an empty graph).
+    auto rows_of = [g](int32_t type) -> int64_t { return type == UG_T_EDGE ? g->E : (type == UG_T_SRC_V ? g->V_total : g->V); };
+    if (!C.data && rows_of(C.type) > 0) return set_error(UG_ERR_INVALID_ARG, "C data is NULL");
 
     // Pass 1: copy ops use one operand; copy_rhs is copy_lhs on B.
     const ug_tensor *opa = nullptr, *opb = nullptr;
@@ -63,7 +66,7 @@ ug_status lower(const ug_graph *g, const ug_op_info *op, Lowered *out) {
         if (!t) continue;
         if (t->type != UG_T_SRC_V && t->type != UG_T_DST_V && t->type != UG_T_EDGE)
             return set_error(UG_ERR_UNSUPPORTED_OP, "an operand the edge_op reads has type NULL");
-        if (!t->data) return set_error(UG_ERR_INVALID_ARG, "operand data is NULL");
+        if (!t->data && rows_of(t->type) > 0) return set_error(UG_ERR_INVALID_ARG, "operand data is NULL");
         if (!(t->width == F || t->width == H || t->width == 1))
             return set_error(UG_ERR_SHAPE, "operand width must be F, H or 1");
         if (t->ld < t->width) return set_error(UG_ERR_SHAPE, "operand ld < width");

@@ -1,0 +1,82 @@
+#!/usr/bin/env python
+"""Summarise ncu output for profiles/ (run here, on the CPU host, after gpurun brings the
+reports back).
+
+  python scripts/ncu_summary.py launches gpurun_out/launches_r1.csv        # kernel shares
+  python scripts/ncu_summary.py full gpurun_out/prof_k_split_r1.ncu-rep     # key metrics
+"""
+import csv
+import io
+import json
+import subprocess
+import sys
+from collections import defaultdict
+
+KEYS = [
+    "gpu__time_duration.sum",
+    "dram__bytes_read.sum",
+    "dram__bytes_write.sum",
+    "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
+    "dram__throughput.avg.pct_of_peak_sustained_elapsed",
+    "lts__t_bytes.sum",
+    "lts__t_sectors_srcunit_tex_op_read.sum",
+    "lts__t_sector_hit_rate.pct",
+    "lts__throughput.avg.pct_of_peak_sustained_elapsed",
+    "l1tex__t_bytes.sum",
+    "l1tex__t_sector_hit_rate.pct",
+    "sm__throughput.avg.pct_of_peak_sustained_elapsed",
+    "sm__warps_active.avg.pct_of_peak_sustained_active",
+    "sm__inst_executed.sum",
+    "launch__registers_per_thread",
+    "launch__grid_size",
+    "launch__block_size",
+    "launch__occupancy_limit_registers",
+    "sm__maximum_warps_per_active_cycle_pct",
+    "smsp__average_warp_latency_issue_stalled_long_scoreboard",
+    "smsp__pcsamp_warps_issue_stalled_long_scoreboard",
+    "smsp__pcsamp_warps_issue_stalled_lg_throttle",
+    "smsp__pcsamp_warps_issue_stalled_wait",
+    "smsp__pcsamp_warps_issue_stalled_selected",
+]
+
+
+def launches(path):
+    lines = open(path).read().splitlines()
+    start = next(i for i, l in enumerate(lines) if l.startswith('"ID"'))
+    rows = list(csv.DictReader(lines[start:]))
+    tot = defaultdict(float)
+    cnt = defaultdict(int)
+    for r in rows:
+        if r.get("Metric Name") != "gpu__time_duration.sum":
+            continue
+        name = r["Kernel Name"].split("(")[0]
+        unit = r.get("Metric Unit", "ns")
+        v = float(r["Metric Value"].replace(",", ""))
+        scale = {"ns": 1e-6, "usecond": 1e-3, "us": 1e-3, "msecond": 1.0, "ms": 1.0, "second": 1e3}.get(unit, 1e-6)
+        tot[name] += v * scale
+        cnt[name] += 1
+    all_ms = sum(tot.values())
+    out = {k: {"launches": cnt[k], "total_ms": round(v, 4), "avg_ms": round(v / cnt[k], 4),
+               "share": round(v / all_ms, 4)} for k, v in sorted(tot.items(), key=lambda kv: -kv[1])}
+    return out
+
+
+def full(path):
+    txt = subprocess.check_output(["ncu", "-i", path, "--page", "raw", "--csv"]).decode()
+    rdr = list(csv.reader(io.StringIO(txt)))
+    hdr, units = rdr[0], rdr[1]
+    res = []
+    for row in rdr[2:]:
+        d = dict(zip(hdr, row))
+        rec = {"kernel": d.get("Kernel Name", "")[:120], "id": d.get("ID")}
+        for k in KEYS:
+            for h in hdr:
+                if h == k:
+                    rec[k] = d[h] + (" " + units[hdr.index(h)] if units[hdr.index(h)] else "")
+        res.append(rec)
+    return res
+
+
+if __name__ == "__main__":
+    mode, path = sys.argv[1], sys.argv[2]
+    print(json.dumps(launches(path) if mode == "launches" else full(path), indent=1))
