@@ -12,7 +12,7 @@
 namespace ug {
 
 template <int KE, int GOP, int VEC>
-__global__ void __launch_bounds__(1024) k_bvertex(GraphArgs g, OpArgs op, int G) {
+__global__ void __launch_bounds__(512) k_bvertex(GraphArgs g, OpArgs op, int G) {
     constexpr int R = (8 / VEC) > 0 ? (8 / VEC) : 1;
     constexpr int CH = 32 * VEC * R;   // features per register block
     extern __shared__ float sm[];      // [NW][CH]
@@ -54,22 +54,7 @@ __global__ void __launch_bounds__(1024) k_bvertex(GraphArgs g, OpArgs op, int G)
                 for (int j = 0; j < R; ++j)
 #pragma unroll
                     for (int i = 0; i < VEC; ++i) acc[j][i] = g_init<GOP>();
-                for (int64_t k = k0 + warp; k < k1; k += NW) {
-                    const int64_t src = g.col[k];
-                    const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
-                    const int64_t ra = op_row(op.A.type, src, v, e);
-                    const int64_t rb = op_row(op.B.type, src, v, e);
-#pragma unroll
-                    for (int j = 0; j < R; ++j) {
-                        const int f = fb0 + j * 32 * VEC + lane * VEC;
-                        if (f < op.W) {
-                            float m[VEC];
-                            message<KE, VEC>(op, ra, ca[j], rb, cb[j], m);
-#pragma unroll
-                            for (int i = 0; i < VEC; ++i) acc[j][i] = g_combine<GOP>(acc[j][i], m[i]);
-                        }
-                    }
-                }
+                gather_row<KE, GOP, VEC, R, 2>(g, op, v, k0 + warp, k1, NW, ca, cb, fb0 + lane * VEC, 32 * VEC, op.W, acc);
 #pragma unroll
                 for (int j = 0; j < R; ++j)
 #pragma unroll

@@ -88,6 +88,67 @@ __device__ __forceinline__ void st_vec(float *p, const float (&r)[VEC]) {
     }
 }
 
+// ---------------------------------------------------------------- L2 cache-policy loads
+// createpolicy + ld.global.nc.L2::cache_hint: keep the gathered feature slab resident
+// (evict_last) while streaming index arrays through L2 (evict_first).
+__device__ __forceinline__ uint64_t l2_policy_evict_last() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_evict_first() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+template <int VEC>
+__device__ __forceinline__ void ldg_vec_hint(const float *__restrict__ p, float (&r)[VEC], uint64_t pol) {
+    if constexpr (VEC == 1) {
+        asm("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(r[0]) : "l"(p), "l"(pol));
+    } else if constexpr (VEC == 2) {
+        asm("ld.global.nc.L2::cache_hint.v2.f32 {%0, %1}, [%2], %3;" : "=f"(r[0]), "=f"(r[1]) : "l"(p), "l"(pol));
+    } else {
+        asm("ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+            : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]) : "l"(p), "l"(pol));
+    }
+}
+
+__device__ __forceinline__ int32_t ldg_i32_hint(const int32_t *__restrict__ p, uint64_t pol) {
+    int32_t r;
+    asm("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+    return r;
+}
+
+template <int VEC>
+__device__ __forceinline__ void fetch_hint(const Operand &x, int64_t row, int64_t col, float (&r)[VEC],
+                                           uint64_t pol) {
+    const float *p = x.p + row * x.ld + col;
+    if (x.div == 1) {
+        ldg_vec_hint<VEC>(p, r, pol);
+    } else {
+        float s = __ldg(p);
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) r[i] = s;
+    }
+}
+
+template <int KE, int VEC>
+__device__ __forceinline__ void message_hint(const OpArgs &op, int64_t ra, int64_t ca, int64_t rb,
+                                             int64_t cb, float (&m)[VEC], uint64_t pol) {
+    float a[VEC];
+    fetch_hint<VEC>(op.A, ra, ca, a, pol);
+    if constexpr (KE == K_COPY) {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) m[i] = a[i];
+    } else {
+        float b[VEC];
+        fetch_hint<VEC>(op.B, rb, cb, b, pol);
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) m[i] = edge_fn<KE>(a[i], b[i]);
+    }
+}
+
 // Store the first n (<= VEC) lanes of a vector: the ragged tail of a row.
 template <int VEC>
 __device__ __forceinline__ void st_vec_n(float *p, const float (&r)[VEC], int n) {
@@ -135,6 +196,57 @@ __device__ __forceinline__ void message(const OpArgs &op, int64_t ra, int64_t ca
         fetch<VEC>(op.B, rb, cb, b);
 #pragma unroll
         for (int i = 0; i < VEC; ++i) m[i] = edge_fn<KE>(a[i], b[i]);
+    }
+}
+
+// Owner-computes gather of one destination row v over in-edge positions k0, k0+kstep, ... < k1
+// into R register chunks of VEC features (chunk j at feature fb + j*stride, valid if < f_hi).
+// U edges are processed per step so that U*R row loads are in flight per lane.
+template <int KE, int GOP, int VEC, int R, int U>
+__device__ __forceinline__ void gather_row(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t k0,
+                                           int64_t k1, int64_t kstep, const int64_t (&ca)[R],
+                                           const int64_t (&cb)[R], int fb, int stride, int f_hi,
+                                           float (&acc)[R][VEC]) {
+    int64_t k = k0;
+    for (; k + (U - 1) * kstep < k1; k += U * kstep) {
+        int64_t ra[U], rb[U];
+#pragma unroll
+        for (int q = 0; q < U; ++q) {
+            const int64_t kk = k + q * kstep;
+            const int64_t src = g.col[kk];
+            const int64_t e = g.eid ? (int64_t)g.eid[kk] : kk;
+            ra[q] = op_row(op.A.type, src, v, e);
+            rb[q] = op_row(op.B.type, src, v, e);
+        }
+#pragma unroll
+        for (int j = 0; j < R; ++j) {
+            const int f = fb + j * stride;
+            if (f < f_hi) {
+                float m[U][VEC];
+#pragma unroll
+                for (int q = 0; q < U; ++q) message<KE, VEC>(op, ra[q], ca[j], rb[q], cb[j], m[q]);
+#pragma unroll
+                for (int q = 0; q < U; ++q)
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) acc[j][i] = g_combine<GOP>(acc[j][i], m[q][i]);
+            }
+        }
+    }
+    for (; k < k1; k += kstep) {
+        const int64_t src = g.col[k];
+        const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
+        const int64_t ra = op_row(op.A.type, src, v, e);
+        const int64_t rb = op_row(op.B.type, src, v, e);
+#pragma unroll
+        for (int j = 0; j < R; ++j) {
+            const int f = fb + j * stride;
+            if (f < f_hi) {
+                float m[VEC];
+                message<KE, VEC>(op, ra, ca[j], rb, cb[j], m);
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) acc[j][i] = g_combine<GOP>(acc[j][i], m[i]);
+            }
+        }
     }
 }
 

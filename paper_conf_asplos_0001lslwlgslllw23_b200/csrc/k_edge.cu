@@ -61,23 +61,60 @@ __global__ void __launch_bounds__(256) k_edge(GraphArgs g, OpArgs op, int L_log2
         } else {
             float acc[R][VEC];
             int64_t cur = -1;
-            for (int64_t k = k0; k < k1; ++k) {
+            auto flush = [&]() {
+#pragma unroll
+                for (int j = 0; j < R; ++j) {
+                    const int f = fb + j * stride;
+                    if (f < f_hi) atomic_flush<GOP, VEC>(op.C + cur * op.c_ld + f, acc[j], op.W - f);
+                }
+            };
+            auto reset = [&]() {
+#pragma unroll
+                for (int j = 0; j < R; ++j)
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) acc[j][i] = g_init<GOP>();
+            };
+            constexpr int U = 4;   // U edges' row gathers in flight per lane
+            int64_t k = k0;
+            for (; k + U <= k1; k += U) {
+                int64_t vq[U], ra[U], rb[U];
+#pragma unroll
+                for (int q = 0; q < U; ++q) {
+                    const int64_t src = g.col[k + q];
+                    vq[q] = (int64_t)g.dst[k + q] - g.r0;
+                    const int64_t e = g.eid ? (int64_t)g.eid[k + q] : k + q;
+                    ra[q] = op_row(op.A.type, src, vq[q], e);
+                    rb[q] = op_row(op.B.type, src, vq[q], e);
+                }
+                float m[U][R][VEC];
+#pragma unroll
+                for (int q = 0; q < U; ++q)
+#pragma unroll
+                    for (int j = 0; j < R; ++j) {
+                        const int f = fb + j * stride;
+                        if (f < f_hi) message<KE, VEC>(op, ra[q], ca[j], rb[q], cb[j], m[q][j]);
+                    }
+#pragma unroll
+                for (int q = 0; q < U; ++q) {
+                    if (vq[q] != cur) {
+                        if (cur >= 0) flush();
+                        cur = vq[q];
+                        reset();
+                    }
+#pragma unroll
+                    for (int j = 0; j < R; ++j)
+#pragma unroll
+                        for (int i = 0; i < VEC; ++i) acc[j][i] = g_combine<GOP>(acc[j][i], m[q][j][i]);
+                }
+            }
+            for (; k < k1; ++k) {
                 const int64_t src = g.col[k];
                 const int64_t v = (int64_t)g.dst[k] - g.r0;
                 const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
                 if (v != cur) {
-                    if (cur >= 0) {
-#pragma unroll
-                        for (int j = 0; j < R; ++j) {
-                            const int f = fb + j * stride;
-                            if (f < f_hi) atomic_flush<GOP, VEC>(op.C + cur * op.c_ld + f, acc[j], op.W - f);
-                        }
-                    }
+                    if (cur >= 0) flush();
                     cur = v;
-#pragma unroll
-                    for (int j = 0; j < R; ++j)
-#pragma unroll
-                        for (int i = 0; i < VEC; ++i) acc[j][i] = g_init<GOP>();
+                    reset();
                 }
                 const int64_t ra = op_row(op.A.type, src, v, e);
                 const int64_t rb = op_row(op.B.type, src, v, e);
@@ -85,10 +122,10 @@ __global__ void __launch_bounds__(256) k_edge(GraphArgs g, OpArgs op, int L_log2
                 for (int j = 0; j < R; ++j) {
                     const int f = fb + j * stride;
                     if (f < f_hi) {
-                        float m[VEC];
-                        message<KE, VEC>(op, ra, ca[j], rb, cb[j], m);
+                        float mm[VEC];
+                        message<KE, VEC>(op, ra, ca[j], rb, cb[j], mm);
 #pragma unroll
-                        for (int i = 0; i < VEC; ++i) acc[j][i] = g_combine<GOP>(acc[j][i], m[i]);
+                        for (int i = 0; i < VEC; ++i) acc[j][i] = g_combine<GOP>(acc[j][i], mm[i]);
                     }
                 }
             }

@@ -63,22 +63,7 @@ __global__ void __launch_bounds__(256) k_vertex(GraphArgs g, OpArgs op, int L_lo
                 for (int j = 0; j < R; ++j)
 #pragma unroll
                     for (int i = 0; i < VEC; ++i) acc[j][i] = g_init<GOP>();
-                for (int64_t k = k0; k < k1; ++k) {
-                    const int64_t src = g.col[k];
-                    const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
-                    const int64_t ra = op_row(op.A.type, src, v, e);
-                    const int64_t rb = op_row(op.B.type, src, v, e);
-#pragma unroll
-                    for (int j = 0; j < R; ++j) {
-                        const int f = fb + j * stride;
-                        if (f < f_hi) {
-                            float m[VEC];
-                            message<KE, VEC>(op, ra, ca[j], rb, cb[j], m);
-#pragma unroll
-                            for (int i = 0; i < VEC; ++i) acc[j][i] = g_combine<GOP>(acc[j][i], m[i]);
-                        }
-                    }
-                }
+gather_row<KE, GOP, VEC, R, 4>(g, op, v, k0, k1, 1, ca, cb, fb, stride, f_hi, acc);
                 const int64_t deg = k1 - k0;
 #pragma unroll
                 for (int j = 0; j < R; ++j) {

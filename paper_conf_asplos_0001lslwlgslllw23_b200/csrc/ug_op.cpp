@@ -135,9 +135,9 @@ ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, La
     const int T = s.tile > 0 ? s.tile : 1;
     if (!is_pow2(T)) return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "tile T must be a power of two");
     c.block = s.block_threads > 0 ? s.block_threads : 256;
-    const int max_block = (c.strategy == UG_BV) ? 1024 : 256;
+    const int max_block = (c.strategy == UG_BV) ? 512 : 256;
     if (c.block % 32 || c.block > max_block)
-        return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "block_threads must be a multiple of 32 and <= 256 (1024 for BV)");
+        return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "block_threads must be a multiple of 32 and <= 256 (512 for BV)");
     // Lanes: lanes beyond the feature chunks of one unit would have no work; they are not
     // launched (clamp rule).
     const int span = lw.dot ? lw.args.D : lw.args.W;
@@ -159,6 +159,7 @@ ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, La
         c.L = L;
     }
     if (c.strategy == UG_BE) c.L = std::min(32, need);
+    if (c.strategy == UG_SV && lw.dot) c.G = 1;   // dot under SV: one row per lane group (k_dot)
     *cfg = c;
     return UG_OK;
 }
