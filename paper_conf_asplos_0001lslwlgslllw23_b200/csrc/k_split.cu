@@ -18,32 +18,26 @@
 
 namespace ug {
 
-template <int KE, int GOP, int VEC>
+template <int KE, int GOP, int VEC, bool FAST>
 __global__ void __launch_bounds__(256) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
                                                int64_t n_chunks, int L_log2, int ftile, int n_tiles,
                                                float *__restrict__ scratch, int64_t sld) {
-    constexpr int U = 8;                       // independent row gathers in flight per lane
-    const int L = 1 << L_log2;
+    constexpr int U = 4;                       // independent row gathers in flight per lane
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const int lane = (int)(t & (L - 1));
+    const int lane = (int)(t & ((1 << L_log2) - 1));
     const int64_t u = t >> L_log2;
-    if (u >= n_chunks * n_tiles) return;       // whole lane groups exit together
+    if (u >= n_chunks * n_tiles) return;
     const int tile = (int)(u / n_chunks);
     const int64_t c = u - (int64_t)tile * n_chunks;
     const int f = tile * ftile + lane * VEC;
-    const bool active = f < op.W;              // idle lanes of a ragged last tile still shuffle
+    if (f >= op.W) return;
     const int4 ch = chunks[c];
     const int64_t v = ch.x;
     const int64_t k1 = ch.z;
-    const int64_t ca = op_col(op.A, active ? f : 0);
-    const int64_t cb = op_col(op.B, active ? f : 0);
-    const unsigned wl = threadIdx.x & 31;
-    const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << (wl & ~(unsigned)(L - 1)));
-    const uint64_t keep = l2_policy_evict_last();    // the X column slab of this tile
-    const uint64_t stream = l2_policy_evict_first(); // col_idx / eid: read once per tile pass
+    const int64_t ca = op_col(op.A, f);
+    const int64_t cb = op_col(op.B, f);
 
     if constexpr (GOP == UG_GATHER_ASSIGN) {
-        if (!active) return;
         for (int64_t k = ch.y; k < k1; ++k) {
             const int64_t src = g.col[k];
             const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
@@ -55,43 +49,57 @@ __global__ void __launch_bounds__(256) k_split(GraphArgs g, OpArgs op, const int
         float acc[VEC];
 #pragma unroll
         for (int i = 0; i < VEC; ++i) acc[i] = g_init<GOP>();
-        // The lane group loads L in-edge indices with one coalesced request, then broadcasts
-        // them by shuffle; each lane keeps U row gathers in flight.
-        for (int64_t kb = ch.y; kb < k1; kb += L) {
-            const int n = (int)(k1 - kb < (int64_t)L ? k1 - kb : (int64_t)L);
-            const int my_src = lane < n ? ldg_i32_hint(g.col + kb + lane, stream) : 0;
-            const int my_e = (g.eid && lane < n) ? ldg_i32_hint(g.eid + kb + lane, stream) : 0;
-            int j = 0;
-            for (; j + U <= n; j += U) {
+        int64_t k = ch.y;
+        if constexpr (FAST) {
+            // A is a full-width Src_V operand and edge ids are CSR positions: the row address is
+            // one IMAD from the (warp-uniform, L1-broadcast) column index.
+            const uint64_t stream = l2_policy_evict_first();   // col_idx: read once per tile pass
+            const float *__restrict__ Ab = op.A.p + f;
+            const int64_t lda = op.A.ld;
+            for (; k + U <= k1; k += U) {
+                int32_t s[U];
+#pragma unroll
+                for (int q = 0; q < U; ++q) s[q] = ldg_i32_hint(g.col + k + q, stream);
+                float m[U][VEC];
+#pragma unroll
+                for (int q = 0; q < U; ++q) ldg_vec<VEC>(Ab + (int64_t)s[q] * lda, m[q]);
+                if constexpr (KE != K_COPY) {
+#pragma unroll
+                    for (int q = 0; q < U; ++q) {
+                        float b[VEC];
+                        fetch<VEC>(op.B, op_row(op.B.type, s[q], v, k + q), cb, b);
+#pragma unroll
+                        for (int i = 0; i < VEC; ++i) m[q][i] = edge_fn<KE>(m[q][i], b[i]);
+                    }
+                }
+#pragma unroll
+                for (int q = 0; q < U; ++q)
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[q][i]);
+            }
+        } else {
+            for (; k + U <= k1; k += U) {
                 float m[U][VEC];
 #pragma unroll
                 for (int q = 0; q < U; ++q) {
-                    const int64_t src = __shfl_sync(gmask, my_src, j + q, L);
-                    const int64_t e = g.eid ? (int64_t)__shfl_sync(gmask, my_e, j + q, L) : kb + j + q;
-                    if (active)
-                        message_hint<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e),
-                                              cb, m[q], keep);
+                    const int64_t src = g.col[k + q];
+                    const int64_t e = g.eid ? (int64_t)g.eid[k + q] : k + q;
+                    message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m[q]);
                 }
-                if (active) {
 #pragma unroll
-                    for (int q = 0; q < U; ++q)
+                for (int q = 0; q < U; ++q)
 #pragma unroll
-                        for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[q][i]);
-                }
-            }
-            for (; j < n; ++j) {
-                const int64_t src = __shfl_sync(gmask, my_src, j, L);
-                const int64_t e = g.eid ? (int64_t)__shfl_sync(gmask, my_e, j, L) : kb + j;
-                if (active) {
-                    float m[VEC];
-                    message_hint<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb,
-                                          m, keep);
-#pragma unroll
-                    for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[i]);
-                }
+                    for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[q][i]);
             }
         }
-        if (!active) return;
+        for (; k < k1; ++k) {
+            const int64_t src = g.col[k];
+            const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
+            float m[VEC];
+            message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m);
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[i]);
+        }
         if (ch.w < 0) {
             const int64_t deg = (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
             float out[VEC];
@@ -142,11 +150,17 @@ cudaError_t launch_split_vertex(int kedge, int gather, const GraphArgs &g, const
     const int64_t sld = cdiv(op.W, 4) * 4;
     const int4 *chunks = reinterpret_cast<const int4 *>(plan.d_chunk);
     if (ev_begin) cudaEventRecord(ev_begin, s);
+    const bool fast = op.A.type == UG_T_SRC_V && op.A.div == 1 && g.eid == nullptr;
     UG_DISPATCH_VEC(c.vec, VEC,
         UG_DISPATCH_KE(kedge, KE,
-            UG_DISPATCH_GOP(gather, GOP,
-                k_split<KE, GOP, VEC><<<(unsigned)grid, c.block, 0, s>>>(
-                    g, op, chunks, plan.n_chunks, L_log2, c.ftile, n_tiles, scratch, sld))));
+            UG_DISPATCH_GOP(gather, GOP, {
+                if (fast)
+                    k_split<KE, GOP, VEC, true><<<(unsigned)grid, c.block, 0, s>>>(
+                        g, op, chunks, plan.n_chunks, L_log2, c.ftile, n_tiles, scratch, sld);
+                else
+                    k_split<KE, GOP, VEC, false><<<(unsigned)grid, c.block, 0, s>>>(
+                        g, op, chunks, plan.n_chunks, L_log2, c.ftile, n_tiles, scratch, sld);
+            })));
     if (ev_end) cudaEventRecord(ev_end, s);
     cudaError_t err = cudaGetLastError();
     if (err != cudaSuccess || gather == UG_GATHER_ASSIGN || plan.n_split_rows == 0) return err;
