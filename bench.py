@@ -148,6 +148,75 @@ def cores_used():
     return 1
 
 
+# Per op x graph latencies on the other BASELINE.json configs (C1-C4): (config, op name,
+# edge_op, gather_op, A type, B type, C type, F, H, A width, B width).
+SECONDARY = [
+    ("C1", "u_mul_e_sum", "mul", "sum", "u", "e", "v", 16, 1, 16, 1),
+    ("C2", "u_add_v", "add", "assign", "u", "v", "e", 8, 8, 8, 8),
+    ("C2", "copy_e_max", "copy_lhs", "max", "e", None, "v", 8, 8, 8, 0),
+    ("C2", "copy_e_sum", "copy_lhs", "sum", "e", None, "v", 8, 8, 8, 0),
+    ("C2", "e_sub_v", "sub", "assign", "e", "v", "e", 8, 8, 8, 8),
+    ("C2", "e_div_v", "div", "assign", "e", "v", "e", 8, 8, 8, 8),
+    ("C2", "u_mul_e_sum", "mul", "sum", "u", "e", "v", 64, 8, 64, 8),
+    ("C3", "copy_u_sum", "copy_lhs", "sum", "u", None, "v", 128, 1, 128, 0),
+    ("C3", "u_mul_e_sum", "mul", "sum", "u", "e", "v", 128, 1, 128, 1),
+    ("C3", "copy_u_sum", "copy_lhs", "sum", "u", None, "v", 32, 1, 32, 0),
+    ("C4", "u_dot_v", "dot", "assign", "u", "v", "e", 128, 1, 128, 128),
+    ("C4", "u_dot_v", "dot", "assign", "u", "v", "e", 256, 1, 256, 256),
+    ("C4", "u_dot_v_H4", "dot", "assign", "u", "v", "e", 128, 4, 128, 128),
+]
+
+
+def secondary_configs(ug, torch, dev, reps=20, warm=5):
+    """Latency (median of `reps` CUDA-event timings after `warm` warm-ups) and effective GB/s,
+    warm L2 (back to back) and cold L2 (a 256 MB scrub written between runs), per op x graph."""
+    import ugdata
+    out = []
+    scrub = torch.empty(64 * 1024 * 1024, device=dev)     # 256 MB > 2 x L2
+    graphs = {}
+    for (cfg, nm, eo, go, a, b, c, F, H, wa, wb) in SECONDARY:
+        if cfg not in graphs:
+            s, d = ugdata.graph(cfg)
+            graphs[cfg] = (ug.Graph(ugdata.CONFIGS[cfg].V, s, d), len(s))
+        g, E = graphs[cfg]
+        V = ugdata.CONFIGS[cfg].V
+        rows = lambda t: V if t in ("u", "v") else E
+        A = torch.rand(rows(a), wa, device=dev) - 0.5
+        B = (torch.rand(rows(b), wb, device=dev) + 0.5) if b else None
+        W = H if eo == "dot" else F
+        C = torch.empty(V if c == "v" else E, W, device=dev)
+        kw = dict(A=A, a_type=a, B=B, b_type=b, C=C, c_type=c, F=F, H=H)
+        sched = ug.schedule_select(g, eo, go, **kw)
+        by = 4 * (V + 1) + 4 * E
+        for t, w in ((a, wa), (b, wb)):
+            if t in ("u", "e"):
+                by += 4 * E * w
+            elif t == "v":
+                by += 4 * V * w
+        by += 4 * (V if c == "v" else E) * W
+        res = {}
+        for mode in ("warm", "cold"):
+            ts = []
+            for i in range(warm + reps):
+                if mode == "cold":
+                    scrub.fill_(float(i))
+                e0 = torch.cuda.Event(enable_timing=True)
+                e1 = torch.cuda.Event(enable_timing=True)
+                e0.record()
+                ug.op_run(g, eo, go, schedule=sched, **kw)
+                e1.record()
+                torch.cuda.synchronize()
+                if i >= warm:
+                    ts.append(e0.elapsed_time(e1))
+            ms = statistics.median(ts)
+            res[mode] = {"latency_us": round(ms * 1e3, 2), "gbs": round(by / (ms * 1e-3) / 1e9, 1)}
+        out.append({"config": cfg, "op": nm, "F": F, "H": H, "schedule": sched, "logical_bytes": by,
+                    "warm": res["warm"], "cold": res["cold"]})
+        del A, B, C
+    del scrub
+    return out
+
+
 # ---------------------------------------------------------------------------- GPU run
 def main():
     ap = argparse.ArgumentParser()
@@ -161,6 +230,7 @@ def main():
     ap.add_argument("--schedule", default=None, help="Table 9 notation; default: ug_schedule_select")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-secondary", action="store_true", help="skip the C1-C4 per op x graph latencies")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -311,6 +381,10 @@ def main():
         except (ValueError, OSError):
             traffic = None
 
+    secondary = None
+    if rank == 0 and world == 1 and not args.no_secondary:
+        secondary = secondary_configs(ug, torch, dev)
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         gbs, nr, ne, dt = oracle_sample(args.config, args.op, F, src, dst, V)
@@ -340,6 +414,7 @@ def main():
             "e2e": e2e,
             "gpu_launches": launches * args.steps,
             "clocks": clocks.summary(),
+            "per_op_graph": secondary,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

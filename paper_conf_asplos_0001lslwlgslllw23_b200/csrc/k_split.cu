@@ -51,29 +51,30 @@ __global__ void __launch_bounds__(256) k_split(GraphArgs g, OpArgs op, const int
         for (int i = 0; i < VEC; ++i) acc[i] = g_init<GOP>();
         int64_t k = ch.y;
         if constexpr (FAST) {
-            // A is a full-width Src_V operand and edge ids are CSR positions: the row address is
-            // one IMAD from the (warp-uniform, L1-broadcast) column index.
-            const uint64_t stream = l2_policy_evict_first();   // col_idx: read once per tile pass
-            const float *__restrict__ Ab = op.A.p + f;
-            const int64_t lda = op.A.ld;
-            for (; k + U <= k1; k += U) {
-                int32_t s[U];
+            // A is a full-width Src_V operand smaller than 4 GiB and edge ids are CSR positions:
+            // the row address is ONE 32x32->64 IMAD.WIDE from the (warp-uniform, L1-broadcast)
+            // column index, so each in-edge costs ~5 instructions per lane.
+            constexpr int UF = 8;
+            const float *__restrict__ Ab = op.A.p;          // warp-uniform base
+            const uint32_t lda = (uint32_t)op.A.ld, fo = (uint32_t)f;
+            for (; k + UF <= k1; k += UF) {
+                uint32_t s[UF];
 #pragma unroll
-                for (int q = 0; q < U; ++q) s[q] = ldg_i32_hint(g.col + k + q, stream);
-                float m[U][VEC];
+                for (int q = 0; q < UF; ++q) s[q] = (uint32_t)__ldg(g.col + k + q);
+                float m[UF][VEC];
 #pragma unroll
-                for (int q = 0; q < U; ++q) ldg_vec<VEC>(Ab + (int64_t)s[q] * lda, m[q]);
+                for (int q = 0; q < UF; ++q) ldg_vec<VEC>(Ab + (s[q] * lda + fo), m[q]);
                 if constexpr (KE != K_COPY) {
 #pragma unroll
-                    for (int q = 0; q < U; ++q) {
+                    for (int q = 0; q < UF; ++q) {
                         float b[VEC];
-                        fetch<VEC>(op.B, op_row(op.B.type, s[q], v, k + q), cb, b);
+                        fetch<VEC>(op.B, op_row(op.B.type, (int64_t)s[q], v, k + q), cb, b);
 #pragma unroll
                         for (int i = 0; i < VEC; ++i) m[q][i] = edge_fn<KE>(m[q][i], b[i]);
                     }
                 }
 #pragma unroll
-                for (int q = 0; q < U; ++q)
+                for (int q = 0; q < UF; ++q)
 #pragma unroll
                     for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[q][i]);
             }
@@ -150,7 +151,10 @@ cudaError_t launch_split_vertex(int kedge, int gather, const GraphArgs &g, const
     const int64_t sld = cdiv(op.W, 4) * 4;
     const int4 *chunks = reinterpret_cast<const int4 *>(plan.d_chunk);
     if (ev_begin) cudaEventRecord(ev_begin, s);
-    const bool fast = op.A.type == UG_T_SRC_V && op.A.div == 1 && g.eid == nullptr;
+    // fast path: full-width Src_V operand whose rows are byte-addressable in 32 bits
+    // (V_total * ld * 4 < 2^32; the host passes the bound in op.A.ld via g.V_src), identity eids
+    const bool fast = op.A.type == UG_T_SRC_V && op.A.div == 1 && g.eid == nullptr &&
+                      (uint64_t)g.V_src * (uint64_t)op.A.ld * 4ull < (1ull << 32);
     UG_DISPATCH_VEC(c.vec, VEC,
         UG_DISPATCH_KE(kedge, KE,
             UG_DISPATCH_GOP(gather, GOP, {

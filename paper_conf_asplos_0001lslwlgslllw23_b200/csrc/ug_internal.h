@@ -30,6 +30,7 @@ struct GraphArgs {
     int64_t E;               // local edges
     int64_t rp_base;         // row_ptr[r0] of a view (0 for a base graph)
     int64_t r0;              // first global row of a view (0 for a base graph)
+    int64_t V_src;           // size of the source-vertex id space (Src_V operand rows)
 };
 
 struct OpArgs {

@@ -174,6 +174,7 @@ static GraphArgs graph_args(const ug_graph *g) {
     a.E = g->E;
     a.rp_base = g->e0;
     a.r0 = g->r0;
+    a.V_src = g->V_total;
     return a;
 }
 

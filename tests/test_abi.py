@@ -211,3 +211,36 @@ def test_launch_counts_follow_pass2():
     Z = torch.zeros(E, 16)
     assert ug.launch_count(g, "add", "assign", A=X, a_type="u", B=X, b_type="v", C=Z, c_type="e",
                            schedule="TE_G1_T16") == 1
+
+
+def test_selector_table_load_and_match(tmp_path):
+    """A measured table entry matching (class, F, degree, CV, V) wins; a miss falls back to the
+    priors; a malformed table is rejected."""
+    src, dst = ugdata.graph("C1")
+    V, E = ugdata.CONFIGS["C1"].V, len(src)
+    g = host_graph(V, src, dst)
+    st = g.stats()
+    t = tmp_path / "table.json"
+    t.write_text('{"version": 1, "entries": [\n'
+                 ' {"class": "agg", "F_lo": 8, "F_hi": 20, "deg_lo": 1, "deg_hi": 10, "cv_lo": 0, "cv_hi": 5,'
+                 '  "V_lo": 1000, "V_hi": 10000, "schedule": "BV_G4_B256"},\n'
+                 ' {"class": "msg", "F_lo": 8, "F_hi": 20, "schedule": "WE_G16_T1"}]}')
+    ug.selector_load(t)
+    X, Y = torch.zeros(V, 16), torch.zeros(V, 16)
+    assert ug.schedule_select(g, "copy_lhs", "sum", A=X, a_type="u", C=Y, c_type="v") == "BV_G4_B256"
+    Z = torch.zeros(E, 16)
+    assert ug.schedule_select(g, "add", "assign", A=X, a_type="u", B=X, b_type="v", C=Z, c_type="e") == "WE_G16_T1"
+    X2, Y2 = torch.zeros(V, 64), torch.zeros(V, 64)     # F outside every entry -> prior
+    assert ug.schedule_select(g, "copy_lhs", "sum", A=X2, a_type="u", C=Y2, c_type="v").startswith("SV")
+    bad = tmp_path / "bad.json"
+    bad.write_text('{"entries": [{"class": "agg", "schedule": "XX_G1"}]}')
+    with pytest.raises(ug.UgError):
+        ug.selector_load(bad)
+    # restore the shipped table (if any) for later tests
+    shipped = os.path.join(ROOT, "paper_conf_asplos_0001lslwlgslllw23_b200", "selector_table.json")
+    if os.path.exists(shipped):
+        ug.selector_load(shipped)
+    else:
+        empty = tmp_path / "empty.json"
+        empty.write_text('{"entries": []}')
+        ug.selector_load(empty)
