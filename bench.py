@@ -169,7 +169,9 @@ SECONDARY = [
 
 def secondary_configs(ug, torch, dev, reps=20, warm=5):
     """Latency (median of `reps` CUDA-event timings after `warm` warm-ups) and effective GB/s,
-    warm L2 (back to back) and cold L2 (a 256 MB scrub written between runs), per op x graph."""
+    warm L2 (back to back) and cold L2 (a 256 MB scrub written between runs), per op x graph.
+    Each timed op is queued behind GPU work so the events measure device time, not the host's
+    launch latency (which is reported separately as host_launch_us)."""
     import ugdata
     out = []
     scrub = torch.empty(64 * 1024 * 1024, device=dev)     # 256 MB > 2 x L2
@@ -199,7 +201,9 @@ def secondary_configs(ug, torch, dev, reps=20, warm=5):
             ts = []
             for i in range(warm + reps):
                 if mode == "cold":
-                    scrub.fill_(float(i))
+                    scrub.fill_(float(i))       # evict L2; also queues the op behind GPU work
+                else:
+                    torch.cuda._sleep(400_000)  # queue behind a spin kernel: device time only
                 e0 = torch.cuda.Event(enable_timing=True)
                 e1 = torch.cuda.Event(enable_timing=True)
                 e0.record()
@@ -210,8 +214,14 @@ def secondary_configs(ug, torch, dev, reps=20, warm=5):
                     ts.append(e0.elapsed_time(e1))
             ms = statistics.median(ts)
             res[mode] = {"latency_us": round(ms * 1e3, 2), "gbs": round(by / (ms * 1e-3) / 1e9, 1)}
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(20):
+            ug.op_run(g, eo, go, schedule=sched, **kw)
+        host_us = (time.perf_counter() - t0) / 20 * 1e6
+        torch.cuda.synchronize()
         out.append({"config": cfg, "op": nm, "F": F, "H": H, "schedule": sched, "logical_bytes": by,
-                    "warm": res["warm"], "cold": res["cold"]})
+                    "warm": res["warm"], "cold": res["cold"], "host_launch_us": round(host_us, 2)})
         del A, B, C
     del scrub
     return out

@@ -199,6 +199,20 @@ __device__ __forceinline__ void message(const OpArgs &op, int64_t ra, int64_t ca
     }
 }
 
+// Message when A is a full-width Src_V operand addressable with 32-bit element offsets
+// (V * ld < 2^32): the row address is one IMAD + IMAD.WIDE from the column index.
+template <int KE, int VEC>
+__device__ __forceinline__ void message_fast(const OpArgs &op, uint32_t src, uint32_t f, int64_t rb,
+                                             int64_t cb, float (&m)[VEC]) {
+    ldg_vec<VEC>(op.A.p + (src * (uint32_t)op.A.ld + f), m);
+    if constexpr (KE != K_COPY) {
+        float b[VEC];
+        fetch<VEC>(op.B, rb, cb, b);
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) m[i] = edge_fn<KE>(m[i], b[i]);
+    }
+}
+
 // Owner-computes gather of one destination row v over in-edge positions k0, k0+kstep, ... < k1
 // into R register chunks of VEC features (chunk j at feature fb + j*stride, valid if < f_hi).
 // U edges are processed per step so that U*R row loads are in flight per lane.

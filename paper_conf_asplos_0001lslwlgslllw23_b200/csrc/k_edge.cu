@@ -16,7 +16,7 @@
 
 namespace ug {
 
-template <int KE, int GOP, int VEC>
+template <int KE, int GOP, int VEC, bool FAST>
 __global__ void __launch_bounds__(256) k_edge(GraphArgs g, OpArgs op, int L_log2, int G,
                                               int ftile, int64_t n_groups, int n_tiles) {
     constexpr int R = (8 / VEC) > 0 ? (8 / VEC) : 1;
@@ -92,7 +92,12 @@ __global__ void __launch_bounds__(256) k_edge(GraphArgs g, OpArgs op, int L_log2
 #pragma unroll
                     for (int j = 0; j < R; ++j) {
                         const int f = fb + j * stride;
-                        if (f < f_hi) message<KE, VEC>(op, ra[q], ca[j], rb[q], cb[j], m[q][j]);
+                        if (f < f_hi) {
+                            if constexpr (FAST)
+                                message_fast<KE, VEC>(op, (uint32_t)ra[q], (uint32_t)f, rb[q], cb[j], m[q][j]);
+                            else
+                                message<KE, VEC>(op, ra[q], ca[j], rb[q], cb[j], m[q][j]);
+                        }
                     }
 #pragma unroll
                 for (int q = 0; q < U; ++q) {
@@ -149,11 +154,18 @@ cudaError_t launch_edge(int kedge, int gather, const GraphArgs &g, const OpArgs 
     if (threads == 0) return cudaSuccess;
     const int64_t grid = cdiv(threads, c.block);
     const int L_log2 = ilog2(c.L);
+    const bool fast = op.A.type == UG_T_SRC_V && op.A.div == 1 &&
+                      (uint64_t)g.V_src * (uint64_t)op.A.ld < (1ull << 32);
     UG_DISPATCH_VEC(c.vec, VEC,
         UG_DISPATCH_KE(kedge, KE,
-            UG_DISPATCH_GOP(gather, GOP,
-                k_edge<KE, GOP, VEC><<<(unsigned)grid, c.block, 0, s>>>(g, op, L_log2, c.G, ft,
-                                                                        n_groups, n_tiles))));
+            UG_DISPATCH_GOP(gather, GOP, {
+                if (fast)
+                    k_edge<KE, GOP, VEC, true><<<(unsigned)grid, c.block, 0, s>>>(g, op, L_log2, c.G, ft,
+                                                                                  n_groups, n_tiles);
+                else
+                    k_edge<KE, GOP, VEC, false><<<(unsigned)grid, c.block, 0, s>>>(g, op, L_log2, c.G, ft,
+                                                                                   n_groups, n_tiles);
+            })));
     return cudaGetLastError();
 }
 

@@ -94,6 +94,9 @@ ug_status lower(const ug_graph *g, const ug_op_info *op, Lowered *out) {
     lw.args.H = H;
     lw.args.D = F / H;
     lw.op_class = dot ? (to_edges ? 2 : 3) : (to_edges ? 0 : 1);
+    // aggregation subclasses for the selector: two-operand sums (4) and max/min (5)
+    if (lw.op_class == 1 && (go == UG_GATHER_MAX || go == UG_GATHER_MIN)) lw.op_class = 5;
+    else if (lw.op_class == 1 && opb) lw.op_class = 4;
 
     // Widest legal feature vector (R22 in DESIGN.md): every full-width operand row must be
     // aligned and either F % vec == 0 or padded (ld >= round_up(F, vec)); a broadcast operand

@@ -19,7 +19,7 @@ struct Lowered {
     OpArgs args;
     int max_vec;        // widest legal feature vector (1, 2, 4)
     // selector key
-    int op_class;       // 0 msg, 1 agg, 2 dot msg, 3 dot agg
+    int op_class;       // 0 msg, 1 agg (copy, sum/mean), 2 dot msg, 3 dot agg, 4 agg_bin, 5 agg_ext
 };
 
 ug_status lower(const ug_graph *g, const ug_op_info *op, Lowered *out);

@@ -38,6 +38,8 @@ static int class_of(const std::string &s) {
     if (s == "agg") return 1;
     if (s == "dot_msg") return 2;
     if (s == "dot_agg") return 3;
+    if (s == "agg_bin") return 4;   // aggregation with two operands (e.g. u_mul_e_sum)
+    if (s == "agg_ext") return 5;   // max / min aggregation
     return -1;
 }
 
@@ -139,7 +141,7 @@ static ug_schedule prior(const ug_graph *g, const Lowered &lw) {
         s.strategy = UG_TE; s.group = 1; s.tile = dl;
     } else if (lw.op_class == 3) {
         s.strategy = UG_WV; s.group = 1; s.tile = 1;
-    } else {                           // aggregation
+    } else {                           // aggregation (classes 1, 4, 5)
         if (W >= 32 || g->max_deg > 256) { s.strategy = UG_SV; s.group = 1024; s.ftile = 0; }
         else { s.strategy = UG_WV; s.group = 1; s.tile = 1; }
     }
@@ -156,15 +158,20 @@ ug_status select_schedule(const ug_graph *g, const Lowered &lw, ug_schedule *out
     }
     const double F = lw.args.F, deg = g->mean_deg, V = (double)g->V;
     const double cv = g->mean_deg > 0 ? g->std_nnz / g->mean_deg : 0.0;
-    for (const Entry &e : g_table) {
-        if (e.op_class != -1 && e.op_class != lw.op_class) continue;
-        if (F < e.F_lo || F > e.F_hi || deg < e.deg_lo || deg > e.deg_hi || cv < e.cv_lo || cv > e.cv_hi ||
-            V < e.V_lo || V > e.V_hi)
-            continue;
-        ug_schedule s = e.sched;
-        if (s.vec > lw.max_vec) s.vec = 0;   // table entry measured on an aligned layout
-        *out = s;
-        return UG_OK;
+    // exact class first, then the parent class (agg_bin / agg_ext -> agg)
+    const int classes[2] = {lw.op_class, (lw.op_class == 4 || lw.op_class == 5) ? 1 : -2};
+    for (int pass = 0; pass < 2; ++pass) {
+        if (classes[pass] == -2) break;
+        for (const Entry &e : g_table) {
+            if (e.op_class != -1 && e.op_class != classes[pass]) continue;
+            if (F < e.F_lo || F > e.F_hi || deg < e.deg_lo || deg > e.deg_hi || cv < e.cv_lo || cv > e.cv_hi ||
+                V < e.V_lo || V > e.V_hi)
+                continue;
+            ug_schedule s = e.sched;
+            if (s.vec > lw.max_vec) s.vec = 0;   // table entry measured on an aligned layout
+            *out = s;
+            return UG_OK;
+        }
     }
     *out = prior(g, lw);
     return UG_OK;

@@ -27,9 +27,9 @@ import ugdata  # noqa: E402
 
 # op class -> representative ops (name, edge_op, gather, A type, B type, C type)
 CLASS_OPS = {
-    "agg": [("copy_u_sum", "copy_lhs", "sum", "u", None, "v"),
-            ("u_mul_e_sum", "mul", "sum", "u", "e", "v"),
-            ("copy_u_max", "copy_lhs", "max", "u", None, "v")],
+    "agg": [("copy_u_sum", "copy_lhs", "sum", "u", None, "v")],
+    "agg_bin": [("u_mul_e_sum", "mul", "sum", "u", "e", "v")],
+    "agg_ext": [("copy_u_max", "copy_lhs", "max", "u", None, "v")],
     "msg": [("u_add_v", "add", "assign", "u", "v", "e")],
     "dot_msg": [("u_dot_v", "dot", "assign", "u", "v", "e")],
     "dot_agg": [("u_dot_v_sum", "dot", "sum", "u", "v", "v")],
@@ -37,25 +37,26 @@ CLASS_OPS = {
 
 # F per config and class (SURVEY 8(d) widths)
 WIDTHS = {
-    "C1": {"agg": [16], "msg": [16], "dot_msg": [16], "dot_agg": [16]},
-    "C2": {"agg": [16, 64], "msg": [8, 64], "dot_msg": [64], "dot_agg": [64]},
-    "C3": {"agg": [32, 64, 128], "msg": [32], "dot_msg": [128], "dot_agg": [64]},
-    "C4": {"agg": [128], "msg": [128], "dot_msg": [128, 256], "dot_agg": [128]},
-    "C5": {"agg": [602], "msg": [1], "dot_msg": [602], "dot_agg": [602]},
+    "C1": {"agg": [16], "agg_bin": [16], "agg_ext": [16], "msg": [16], "dot_msg": [16], "dot_agg": [16]},
+    "C2": {"agg": [8, 64], "agg_bin": [64], "agg_ext": [8, 64], "msg": [8, 64], "dot_msg": [64], "dot_agg": [64]},
+    "C3": {"agg": [32, 64, 128], "agg_bin": [32, 128], "agg_ext": [32, 128], "msg": [32], "dot_msg": [128],
+           "dot_agg": [64]},
+    "C4": {"agg": [128], "agg_bin": [128], "agg_ext": [128], "msg": [128], "dot_msg": [128, 256], "dot_agg": [128]},
+    "C5": {"agg": [602], "agg_bin": [602], "agg_ext": [602], "msg": [1], "dot_msg": [602], "dot_agg": [602]},
 }
 
 
 def candidates(cls, F, E, quick=False):
     c = []
     Ts = [t for t in (1, 2, 4, 8, 16, 32) if t <= max(1, F)]
-    if cls in ("agg", "dot_agg"):
+    if cls in ("agg", "agg_bin", "agg_ext", "dot_agg"):
         c += [f"TV_G{g}_T{t}" for g in (1, 4) for t in Ts]
         c += [f"WV_G{g}_T1" for g in (1, 2, 8)]
         c += [f"TE_G{g}_T{t}" for g in (1, 8, 32) for t in Ts if t >= 4]
         c += [f"WE_G{g}_T1" for g in (4, 32, 128)]
         c += [f"BV_G{g}_B{b}" for g in (1, 4) for b in (128, 256, 512)]
         c += [f"BE_G{g}" for g in (64, 512)]
-        if cls == "agg":
+        if cls != "dot_agg":
             fts = [f for f in (16, 32, 64, 128) if f <= max(16, 2 * F)]
             c += [f"SV_G{g}_F{f}" for g in (128, 512, 1024, 2048, 4096) for f in fts]
         else:
@@ -68,7 +69,8 @@ def candidates(cls, F, E, quick=False):
         c += ["BV_G1_B256", "BE_G256"]
         c += [f"SV_G{g}" for g in (64, 512)]
     if E > 50_000_000:   # C5: drop the schedules that take seconds (atomic per-element TE at F=602)
-        c = [s for s in c if not (s.startswith("TE") and cls == "agg") and not s.startswith("TV_G4")]
+        c = [s for s in c if not (s.startswith("TE") and cls.startswith("agg")) and not s.startswith("TV")
+             and not s.startswith("WV")]
     if quick:
         c = c[::3]
     return c
@@ -84,7 +86,8 @@ def time_schedule(g, kw, eo, go, sched, reps):
         return None, str(e)
     ts = []
     for i in range(reps):
-        ev[2 * i].record()
+        torch.cuda._sleep(400_000)      # queue the op behind a spin kernel: device time only,
+        ev[2 * i].record()              # no host launch latency inside the events
         ug.op_run(g, eo, go, schedule=sched, **kw)
         ev[2 * i + 1].record()
     torch.cuda.synchronize()
