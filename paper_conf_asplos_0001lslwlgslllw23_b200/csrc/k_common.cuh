@@ -114,6 +114,19 @@ __device__ __forceinline__ void ldg_vec_hint(const float *__restrict__ p, float 
     }
 }
 
+template <int VEC>
+__device__ __forceinline__ void st_vec_hint(float *p, const float (&r)[VEC], uint64_t pol) {
+    if constexpr (VEC == 1) {
+        asm volatile("st.global.L2::cache_hint.f32 [%0], %1, %2;" ::"l"(p), "f"(r[0]), "l"(pol) : "memory");
+    } else if constexpr (VEC == 2) {
+        asm volatile("st.global.L2::cache_hint.v2.f32 [%0], {%1, %2}, %3;" ::"l"(p), "f"(r[0]), "f"(r[1]), "l"(pol)
+                     : "memory");
+    } else {
+        asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p), "f"(r[0]), "f"(r[1]),
+                     "f"(r[2]), "f"(r[3]), "l"(pol) : "memory");
+    }
+}
+
 __device__ __forceinline__ int32_t ldg_i32_hint(const int32_t *__restrict__ p, uint64_t pol) {
     int32_t r;
     asm("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));

@@ -18,6 +18,57 @@
 
 namespace ug {
 
+// Inner in-edge loop of the SV fast path.  BM: 0 no B operand, 1 B is Dst_V (constant over
+// the row: loaded once), 2 B is an Edge tensor (row = CSR position), 3 B is Src_V.  All offsets
+// are 32-bit (the host checks rows * ld < 2^32).  Advances k to the last multiple of 8.
+template <int KE, int GOP, int VEC, int BM>
+__device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t &k,
+                                                int64_t k1, int f, int64_t cb, float (&acc)[VEC]) {
+    constexpr int UF = 8;
+    const float *__restrict__ Ab = op.A.p;          // warp-uniform base
+    const uint64_t keep = l2_policy_evict_last();     // this tile's X column slab
+    const uint64_t stream = l2_policy_evict_first();  // col_idx / edge tensors: read once per pass
+    const uint32_t lda = (uint32_t)op.A.ld, fo = (uint32_t)f;
+    const uint32_t ldb = (uint32_t)op.B.ld, cbo = (uint32_t)cb;
+    const bool bfull = op.B.div == 1;
+    float bconst[VEC];
+    if constexpr (BM == 1) fetch<VEC>(op.B, v, cb, bconst);
+    for (; k + UF <= k1; k += UF) {
+        uint32_t s[UF];
+#pragma unroll
+        for (int q = 0; q < UF; ++q) s[q] = (uint32_t)ldg_i32_hint(g.col + k + q, stream);
+        float m[UF][VEC];
+#pragma unroll
+        for (int q = 0; q < UF; ++q) ldg_vec_hint<VEC>(Ab + (s[q] * lda + fo), m[q], keep);
+        if constexpr (BM != 0) {
+#pragma unroll
+            for (int q = 0; q < UF; ++q) {
+                float b[VEC];
+                if constexpr (BM == 1) {
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) b[i] = bconst[i];
+                } else {
+                    const uint32_t row = BM == 2 ? (uint32_t)(k + q) : s[q];
+                    const float *bp = op.B.p + (row * ldb + cbo);
+                    if (bfull) {
+                        ldg_vec_hint<VEC>(bp, b, BM == 2 ? stream : keep);
+                    } else {
+                        const float x = __ldg(bp);
+#pragma unroll
+                        for (int i = 0; i < VEC; ++i) b[i] = x;
+                    }
+                }
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) m[q][i] = edge_fn<KE>(m[q][i], b[i]);
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < UF; ++q)
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[q][i]);
+    }
+}
+
 template <int KE, int GOP, int VEC, bool FAST>
 __global__ void __launch_bounds__(256) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
                                                int64_t n_chunks, int L_log2, int ftile, int n_tiles,
@@ -52,31 +103,15 @@ __global__ void __launch_bounds__(256) k_split(GraphArgs g, OpArgs op, const int
         int64_t k = ch.y;
         if constexpr (FAST) {
             // A is a full-width Src_V operand smaller than 4 GiB and edge ids are CSR positions:
-            // the row address is ONE 32x32->64 IMAD.WIDE from the (warp-uniform, L1-broadcast)
-            // column index, so each in-edge costs ~5 instructions per lane.
-            constexpr int UF = 8;
-            const float *__restrict__ Ab = op.A.p;          // warp-uniform base
-            const uint32_t lda = (uint32_t)op.A.ld, fo = (uint32_t)f;
-            for (; k + UF <= k1; k += UF) {
-                uint32_t s[UF];
-#pragma unroll
-                for (int q = 0; q < UF; ++q) s[q] = (uint32_t)__ldg(g.col + k + q);
-                float m[UF][VEC];
-#pragma unroll
-                for (int q = 0; q < UF; ++q) ldg_vec<VEC>(Ab + (s[q] * lda + fo), m[q]);
-                if constexpr (KE != K_COPY) {
-#pragma unroll
-                    for (int q = 0; q < UF; ++q) {
-                        float b[VEC];
-                        fetch<VEC>(op.B, op_row(op.B.type, (int64_t)s[q], v, k + q), cb, b);
-#pragma unroll
-                        for (int i = 0; i < VEC; ++i) m[q][i] = edge_fn<KE>(m[q][i], b[i]);
-                    }
-                }
-#pragma unroll
-                for (int q = 0; q < UF; ++q)
-#pragma unroll
-                    for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[q][i]);
+            // the row address is one IMAD + IMAD.WIDE from the (warp-uniform, L1-broadcast)
+            // column index, so each in-edge costs ~6 instructions per lane.  The B operand's
+            // addressing mode is resolved once per unit (a Dst_V operand is loaded once).
+            const int bm = KE == K_COPY ? 0 : (op.B.type == UG_T_DST_V ? 1 : (op.B.type == UG_T_EDGE ? 2 : 3));
+            switch (bm) {
+            case 0: split_fast_loop<KE, GOP, VEC, 0>(g, op, v, k, k1, f, cb, acc); break;
+            case 1: split_fast_loop<KE, GOP, VEC, 1>(g, op, v, k, k1, f, cb, acc); break;
+            case 2: split_fast_loop<KE, GOP, VEC, 2>(g, op, v, k, k1, f, cb, acc); break;
+            default: split_fast_loop<KE, GOP, VEC, 3>(g, op, v, k, k1, f, cb, acc); break;
             }
         } else {
             for (; k + U <= k1; k += U) {
@@ -101,14 +136,17 @@ __global__ void __launch_bounds__(256) k_split(GraphArgs g, OpArgs op, const int
 #pragma unroll
             for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[i]);
         }
+        // outputs are written once: evict_first keeps them from displacing the X slab in L2
+        const uint64_t wpol = l2_policy_evict_first();
         if (ch.w < 0) {
             const int64_t deg = (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
             float out[VEC];
 #pragma unroll
             for (int i = 0; i < VEC; ++i) out[i] = g_finalize<GOP>(acc[i], deg);
-            st_vec_n<VEC>(op.C + v * op.c_ld + f, out, op.W - f);
+            if (f + VEC <= op.W) st_vec_hint<VEC>(op.C + v * op.c_ld + f, out, wpol);
+            else st_vec_n<VEC>(op.C + v * op.c_ld + f, out, op.W - f);
         } else {
-            st_vec<VEC>(scratch + (int64_t)ch.w * sld + f, acc);
+            st_vec_hint<VEC>(scratch + (int64_t)ch.w * sld + f, acc, wpol);
         }
     }
 }
@@ -153,8 +191,15 @@ cudaError_t launch_split_vertex(int kedge, int gather, const GraphArgs &g, const
     if (ev_begin) cudaEventRecord(ev_begin, s);
     // fast path: full-width Src_V operand whose rows are byte-addressable in 32 bits
     // (V_total * ld * 4 < 2^32; the host passes the bound in op.A.ld via g.V_src), identity eids
-    const bool fast = op.A.type == UG_T_SRC_V && op.A.div == 1 && g.eid == nullptr &&
-                      (uint64_t)g.V_src * (uint64_t)op.A.ld * 4ull < (1ull << 32);
+    // fast path: full-width Src_V A operand, identity edge ids, and every operand row
+    // addressable with 32-bit element offsets (rows * ld < 2^32)
+    const uint64_t lim = 1ull << 32;
+    bool fast = op.A.type == UG_T_SRC_V && op.A.div == 1 && g.eid == nullptr &&
+                (uint64_t)g.V_src * (uint64_t)op.A.ld < lim;
+    if (kedge != K_COPY) {
+        const uint64_t brows = op.B.type == UG_T_EDGE ? (uint64_t)g.E : (uint64_t)g.V_src;
+        fast = fast && brows * (uint64_t)op.B.ld < lim;
+    }
     UG_DISPATCH_VEC(c.vec, VEC,
         UG_DISPATCH_KE(kedge, KE,
             UG_DISPATCH_GOP(gather, GOP, {

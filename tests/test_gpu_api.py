@@ -1,0 +1,86 @@
+"""GPU tests of the public Python API around ug_op_run: the streamed (host-to-host) pipeline,
+the sharded operator at world size 1, the measurement hook and the selector's choices."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import ugdata
+from gpu_util import assert_parity
+
+pytestmark = pytest.mark.gpu
+
+ug = pytest.importorskip("paper_conf_asplos_0001lslwlgslllw23_b200")
+from paper_conf_asplos_0001lslwlgslllw23_b200.pipeline import StreamedOperator  # noqa: E402
+from paper_conf_asplos_0001lslwlgslllw23_b200.shard import ShardedOperator, x_block  # noqa: E402
+
+
+@pytest.fixture(scope="module")
+def c3():
+    c = ugdata.CONFIGS["C3"]
+    src, dst = ugdata.graph("C3")
+    return c.V, src, dst, ug.Graph(c.V, src, dst)
+
+
+def test_streamed_operator_matches_oracle(c3):
+    V, src, dst, g = c3
+    F = 32
+    Xs = [ugdata.values(V, F, 50 + i, 1, mode="int") for i in range(4)]
+    hin = [torch.from_numpy(x).pin_memory() for x in Xs]
+    hout = [torch.empty(V, F).pin_memory() for _ in Xs]
+    so = StreamedOperator(g, "copy_lhs", "sum", a_type="u", in_shape=(V, F), out_shape=(V, F), depth=2, F=F)
+    so.run(hin, hout)
+    so.synchronize()
+    for x, y in zip(Xs, hout):
+        ref = oracle.op(V, src, dst, "copy_lhs", "sum", A=x, a_type="u", F=F)
+        np.testing.assert_array_equal(y.numpy(), ref)   # integer mode: exact
+
+
+def test_sharded_operator_world1(c3):
+    V, src, dst, g = c3
+    sh = ShardedOperator(g, 1, 0)
+    X = torch.from_numpy(ugdata.values(V, 16, 3, 1, mode="int")).cuda()
+    Y = torch.empty(V, 16, device="cuda")
+    sh.run("copy_lhs", "max", x_block(X, V, 1, 0), Y)
+    Y2 = torch.empty(V, 16, device="cuda")
+    ug.op_run(g, "copy_lhs", "max", A=X, a_type="u", C=Y2, c_type="v")
+    torch.cuda.synchronize()
+    assert torch.equal(Y, Y2)
+
+
+def test_op_run_events_times_main_kernel(c3):
+    V, src, dst, g = c3
+    X = torch.randn(V, 64, device="cuda")
+    Y = torch.empty(V, 64, device="cuda")
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record()
+    e1.record()
+    for sch in ("SV_G512", "TE_G8_T8", "WV_G1_T1", "BV_G1"):
+        ug.op_run_events(g, "copy_lhs", "mean", e0, e1, A=X, a_type="u", C=Y, c_type="v", schedule=sch)
+        torch.cuda.synchronize()
+        assert e0.elapsed_time(e1) > 0.0
+
+
+def test_auto_selection_is_valid_for_every_class(c3):
+    V, src, dst, g = c3
+    E = len(src)
+    X = torch.randn(V, 32, device="cuda")
+    w = torch.rand(E, 1, device="cuda") + 0.5
+    cases = [("copy_lhs", "sum", dict(A=X, a_type="u"), (V, 32), "v"),
+             ("mul", "sum", dict(A=X, a_type="u", B=w, b_type="e"), (V, 32), "v"),
+             ("copy_lhs", "max", dict(A=X, a_type="u"), (V, 32), "v"),
+             ("add", "assign", dict(A=X, a_type="u", B=X, b_type="v"), (E, 32), "e"),
+             ("dot", "assign", dict(A=X, a_type="u", B=X, b_type="v"), (E, 1), "e"),
+             ("dot", "sum", dict(A=X, a_type="u", B=X, b_type="v"), (V, 1), "v")]
+    for eo, go, kw, shape, ct in cases:
+        C = torch.empty(*shape, device="cuda")
+        s = ug.schedule_select(g, eo, go, C=C, c_type=ct, F=32, H=1, **kw)
+        ug.op_run(g, eo, go, C=C, c_type=ct, F=32, H=1, **kw)        # AUTO
+        C2 = torch.empty_like(C)
+        ug.op_run(g, eo, go, C=C2, c_type=ct, F=32, H=1, schedule=s, **kw)
+        torch.cuda.synchronize()
+        if go in ("max", "assign"):
+            assert torch.equal(C, C2), (eo, go, s)
+        else:
+            torch.testing.assert_close(C, C2, rtol=1e-5, atol=1e-5)
