@@ -387,7 +387,9 @@ def main():
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
         try:
-            traffic = json.load(open(tp)).get(f"{args.config}:{args.op}:{F}:{chosen}")
+            ent = json.load(open(tp)).get(f"{args.config}:{args.op}:{F}:{chosen}")
+            # dram__bytes_read.sum + dram__bytes_write.sum of one launch (ncu --set full)
+            traffic = int(ent["dram_bytes_per_launch"]) if ent and world == 1 else None
         except (ValueError, OSError):
             traffic = None
 

@@ -7,7 +7,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libugraph.so")
+LIB_PATH = os.environ.get("UG_LIBRARY") or os.path.join(_HERE, "libugraph.so")   # override: experiments only
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libugraph.so not built at {LIB_PATH}: run `make` in the repo root "

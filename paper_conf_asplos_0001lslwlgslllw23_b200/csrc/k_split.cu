@@ -24,7 +24,8 @@ namespace ug {
 template <int KE, int GOP, int VEC, int BM>
 __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t &k,
                                                 int64_t k1, int f, int64_t cb, float (&acc)[VEC]) {
-    constexpr int UF = 8;
+    // row gathers in flight per lane: 16 (measured +3 % over 8 on C5 at VEC 2), 8 for float4 rows
+    constexpr int UF = VEC == 4 ? 8 : 16;
     const float *__restrict__ Ab = op.A.p;          // warp-uniform base
     const uint64_t keep = l2_policy_evict_last();     // this tile's X column slab
     const uint64_t stream = l2_policy_evict_first();  // col_idx / edge tensors: read once per pass
