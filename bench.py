@@ -220,8 +220,15 @@ def secondary_configs(ug, torch, dev, reps=20, warm=5):
             ug.op_run(g, eo, go, schedule=sched, **kw)
         host_us = (time.perf_counter() - t0) / 20 * 1e6
         torch.cuda.synchronize()
+        pop = ug.prepare(g, eo, go, schedule=sched, **kw)     # marshalled once (serving loop)
+        t0 = time.perf_counter()
+        for _ in range(20):
+            pop()
+        prep_us = (time.perf_counter() - t0) / 20 * 1e6
+        torch.cuda.synchronize()
         out.append({"config": cfg, "op": nm, "F": F, "H": H, "schedule": sched, "logical_bytes": by,
-                    "warm": res["warm"], "cold": res["cold"], "host_launch_us": round(host_us, 2)})
+                    "warm": res["warm"], "cold": res["cold"], "host_launch_us": round(host_us, 2),
+                    "host_launch_prepared_us": round(prep_us, 2)})
         del A, B, C
     del scrub
     return out

@@ -19,7 +19,7 @@ from . import _ffi
 from ._ffi import (EDGE_OPS, GATHER_OPS, STRATEGIES, TTYPES, UgError, UgOpInfo, UgSchedule,
                    UgTensor, check, lib)
 
-__all__ = ["Graph", "op_run", "schedule_select", "launch_count", "parse_schedule",
+__all__ = ["Graph", "op_run", "prepare", "PreparedOp", "schedule_select", "launch_count", "parse_schedule",
            "format_schedule", "validate", "edge_permute", "selector_load", "UgError", "version"]
 
 
@@ -202,6 +202,39 @@ def op_run_events(graph, edge_op, gather_op, ev_begin, ev_end, A=None, a_type=No
                                ctypes.c_void_p(ev_begin.cuda_event), ctypes.c_void_p(ev_end.cuda_event)),
           "ug_op_run_events")
     return C
+
+
+class PreparedOp:
+    """An op_run call with its op_info / parallel_info marshalled once (serving loops, CUDA-graph
+    capture).  The tensors' storage must stay alive and in place; call it like op_run."""
+
+    def __init__(self, graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, C=None,
+                 c_type="v", F=None, H=None, schedule=None):
+        self.info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+        check(lib.ug_op_validate(graph.handle, ctypes.byref(self.info)), "ug_op_validate")
+        if schedule is None:
+            self.sched = UgSchedule()
+            check(lib.ug_schedule_select(graph.handle, ctypes.byref(self.info), ctypes.byref(self.sched)),
+                  "ug_schedule_select")
+        elif isinstance(schedule, UgSchedule):
+            self.sched = schedule
+        else:
+            self.sched = parse_schedule(schedule)
+        self.schedule = format_schedule(self.sched)
+        self._keep = (graph, A, B, C)
+        self._h = graph.handle
+        self._iref = ctypes.byref(self.info)
+        self._sref = ctypes.byref(self.sched)
+
+    def __call__(self, stream=None):
+        st = lib.ug_op_run(self._h, self._iref, self._sref, _current_stream(stream))
+        if st != _ffi.UG_OK:
+            raise UgError(st, "ug_op_run")
+
+
+def prepare(graph, edge_op, gather_op, **kw):
+    """PreparedOp factory: same arguments as op_run (schedule=None resolves AUTO once)."""
+    return PreparedOp(graph, edge_op, gather_op, **kw)
 
 
 def validate(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, C=None, c_type="v",

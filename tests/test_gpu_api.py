@@ -84,3 +84,48 @@ def test_auto_selection_is_valid_for_every_class(c3):
             assert torch.equal(C, C2), (eo, go, s)
         else:
             torch.testing.assert_close(C, C2, rtol=1e-5, atol=1e-5)
+
+
+def test_prepared_op_and_cuda_graph_capture():
+    """PreparedOp == op_run; a GAT-style op chain captured into one CUDA graph replays to the
+    same bits (plans / scratch are stream-ordered, so ug_op_run is capture-safe after warm-up)."""
+    c = ugdata.CONFIGS["C2"]
+    src, dst = ugdata.graph("C2")
+    g = ug.Graph(c.V, src, dst)
+    V, E, H, F = c.V, len(src), 8, 64
+    X = torch.randn(V, F, device="cuda")
+    el = torch.randn(V, H, device="cuda")
+    er = torch.randn(V, H, device="cuda")
+    a = torch.empty(E, H, device="cuda")
+    m = torch.empty(V, H, device="cuda")
+    s = torch.empty(E, H, device="cuda")
+    den = torch.empty(V, H, device="cuda")
+    p = torch.empty(E, H, device="cuda")
+    Y = torch.empty(V, F, device="cuda")
+    chain = [ug.prepare(g, "add", "assign", A=el, a_type="u", B=er, b_type="v", C=a, c_type="e", F=H, H=H),
+             ug.prepare(g, "copy_lhs", "max", A=a, a_type="e", C=m, c_type="v", F=H, H=H),
+             ug.prepare(g, "sub", "assign", A=a, a_type="e", B=m, b_type="v", C=s, c_type="e", F=H, H=H),
+             ug.prepare(g, "copy_lhs", "sum", A=s, a_type="e", C=den, c_type="v", F=H, H=H),
+             ug.prepare(g, "div", "assign", A=s, a_type="e", B=den, b_type="v", C=p, c_type="e", F=H, H=H),
+             ug.prepare(g, "mul", "sum", A=X, a_type="u", B=p, b_type="e", C=Y, c_type="v", F=F, H=H)]
+    side = torch.cuda.Stream()
+    with torch.cuda.stream(side):
+        for op in chain:          # warm-up: plans are built outside the capture
+            op()
+    torch.cuda.synchronize()
+    ref = Y.clone()
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph):
+        for op in chain:
+            op()
+    Y.zero_()
+    graph.replay()
+    torch.cuda.synchronize()
+    # sums may use atomic schedules (order-dependent rounding): tolerance, not bits
+    torch.testing.assert_close(Y, ref, rtol=1e-5, atol=1e-5)
+    # and the chain matches op_run through the public API, op by op
+    Y2 = torch.empty_like(Y)
+    ug.op_run(g, "mul", "sum", A=X, a_type="u", B=p, b_type="e", C=Y2, c_type="v", F=F, H=H,
+              schedule=chain[-1].schedule)
+    torch.cuda.synchronize()
+    torch.testing.assert_close(Y2, ref, rtol=1e-5, atol=1e-5)
