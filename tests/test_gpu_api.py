@@ -94,8 +94,8 @@ def test_prepared_op_and_cuda_graph_capture():
     g = ug.Graph(c.V, src, dst)
     V, E, H, F = c.V, len(src), 8, 64
     X = torch.randn(V, F, device="cuda")
-    el = torch.randn(V, H, device="cuda")
-    er = torch.randn(V, H, device="cuda")
+    el = torch.rand(V, H, device="cuda") + 0.5      # positive: every ratio below is finite
+    er = torch.rand(V, H, device="cuda") + 0.5
     a = torch.empty(E, H, device="cuda")
     m = torch.empty(V, H, device="cuda")
     s = torch.empty(E, H, device="cuda")
@@ -104,7 +104,7 @@ def test_prepared_op_and_cuda_graph_capture():
     Y = torch.empty(V, F, device="cuda")
     chain = [ug.prepare(g, "add", "assign", A=el, a_type="u", B=er, b_type="v", C=a, c_type="e", F=H, H=H),
              ug.prepare(g, "copy_lhs", "max", A=a, a_type="e", C=m, c_type="v", F=H, H=H),
-             ug.prepare(g, "sub", "assign", A=a, a_type="e", B=m, b_type="v", C=s, c_type="e", F=H, H=H),
+             ug.prepare(g, "div", "assign", A=a, a_type="e", B=m, b_type="v", C=s, c_type="e", F=H, H=H),
              ug.prepare(g, "copy_lhs", "sum", A=s, a_type="e", C=den, c_type="v", F=H, H=H),
              ug.prepare(g, "div", "assign", A=s, a_type="e", B=den, b_type="v", C=p, c_type="e", F=H, H=H),
              ug.prepare(g, "mul", "sum", A=X, a_type="u", B=p, b_type="e", C=Y, c_type="v", F=F, H=H)]
@@ -121,6 +121,7 @@ def test_prepared_op_and_cuda_graph_capture():
     Y.zero_()
     graph.replay()
     torch.cuda.synchronize()
+    assert torch.isfinite(ref).all() and ref.abs().sum() > 0
     # sums may use atomic schedules (order-dependent rounding): tolerance, not bits
     torch.testing.assert_close(Y, ref, rtol=1e-5, atol=1e-5)
     # and the chain matches op_run through the public API, op by op
