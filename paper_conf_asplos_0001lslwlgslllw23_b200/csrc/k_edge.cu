@@ -74,10 +74,15 @@ __global__ void __launch_bounds__(256) k_edge(GraphArgs g, OpArgs op, int L_log2
 #pragma unroll
                     for (int i = 0; i < VEC; ++i) acc[j][i] = g_init<GOP>();
             };
-            constexpr int U = 4;   // U edges' row gathers in flight per lane
+            // U edges' row gathers in flight per lane; fewer when each edge already needs
+            // several register chunks (keeps registers, hence occupancy, in check)
+            constexpr int U = (R * VEC >= 8) ? 2 : 4;
+            // a width-1 B operand (e.g. GCN's scalar edge weight) is loaded once per edge
+            const bool bscalar = KE != K_COPY && op.B.div == op.F;
             int64_t k = k0;
             for (; k + U <= k1; k += U) {
                 int64_t vq[U], ra[U], rb[U];
+                float bs[U];
 #pragma unroll
                 for (int q = 0; q < U; ++q) {
                     const int64_t src = g.col[k + q];
@@ -85,6 +90,7 @@ __global__ void __launch_bounds__(256) k_edge(GraphArgs g, OpArgs op, int L_log2
                     const int64_t e = g.eid ? (int64_t)g.eid[k + q] : k + q;
                     ra[q] = op_row(op.A.type, src, vq[q], e);
                     rb[q] = op_row(op.B.type, src, vq[q], e);
+                    if constexpr (KE != K_COPY) bs[q] = bscalar ? __ldg(op.B.p + rb[q] * op.B.ld) : 0.0f;
                 }
                 float m[U][R][VEC];
 #pragma unroll
@@ -93,10 +99,19 @@ __global__ void __launch_bounds__(256) k_edge(GraphArgs g, OpArgs op, int L_log2
                     for (int j = 0; j < R; ++j) {
                         const int f = fb + j * stride;
                         if (f < f_hi) {
-                            if constexpr (FAST)
+                            if constexpr (FAST && KE != K_COPY) {
+                                if (bscalar) {
+                                    ldg_vec<VEC>(op.A.p + ((uint32_t)ra[q] * (uint32_t)op.A.ld + (uint32_t)f), m[q][j]);
+#pragma unroll
+                                    for (int i = 0; i < VEC; ++i) m[q][j][i] = edge_fn<KE>(m[q][j][i], bs[q]);
+                                } else {
+                                    message_fast<KE, VEC>(op, (uint32_t)ra[q], (uint32_t)f, rb[q], cb[j], m[q][j]);
+                                }
+                            } else if constexpr (FAST) {
                                 message_fast<KE, VEC>(op, (uint32_t)ra[q], (uint32_t)f, rb[q], cb[j], m[q][j]);
-                            else
+                            } else {
                                 message<KE, VEC>(op, ra[q], ca[j], rb[q], cb[j], m[q][j]);
+                            }
                         }
                     }
 #pragma unroll

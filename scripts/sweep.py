@@ -54,6 +54,9 @@ def candidates(cls, F, E, quick=False):
         c += [f"WV_G{g}_T1" for g in (1, 2, 8)]
         c += [f"TE_G{g}_T{t}" for g in (1, 8, 32) for t in Ts if t >= 4]
         c += [f"WE_G{g}_T1" for g in (4, 32, 128)]
+        vec = 4 if F % 4 == 0 else (2 if F % 2 == 0 else 1)
+        # edge-parallel with tile-major column tiles (L2 residency of the gathered slab)
+        c += [f"TE_G{g}_T{ft // vec}_F{ft}" for g in (8, 32) for ft in (32, 64) if ft < F and ft // vec <= 32]
         c += [f"BV_G{g}_B{b}" for g in (1, 4) for b in (128, 256, 512)]
         c += [f"BE_G{g}" for g in (64, 512)]
         if cls != "dot_agg":
@@ -69,7 +72,7 @@ def candidates(cls, F, E, quick=False):
         c += ["BV_G1_B256", "BE_G256"]
         c += [f"SV_G{g}" for g in (64, 512)]
     if E > 50_000_000:   # C5: drop the schedules that take seconds (atomic per-element TE at F=602)
-        c = [s for s in c if not (s.startswith("TE") and cls.startswith("agg")) and not s.startswith("TV")
+        c = [s for s in c if not (s.startswith("TE") and cls.startswith("agg") and "_F" not in s) and not s.startswith("TV")
              and not s.startswith("WV")]
     if quick:
         c = c[::3]
