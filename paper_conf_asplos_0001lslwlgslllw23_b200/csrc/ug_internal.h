@@ -74,9 +74,6 @@ cudaError_t launch_block_vertex(int kedge, int gather, const GraphArgs &g, const
 cudaError_t launch_split_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
                                 const LaunchCfg &c, const SplitPlan &plan, float *scratch,
                                 cudaStream_t s, cudaEvent_t ev_begin = nullptr, cudaEvent_t ev_end = nullptr);
-cudaError_t launch_split_dot(int gather, const GraphArgs &g, const OpArgs &op, const LaunchCfg &c,
-                             const SplitPlan &plan, cudaStream_t s, cudaEvent_t ev_begin = nullptr,
-                             cudaEvent_t ev_end = nullptr);
 cudaError_t launch_dot(bool vertex_units, int gather, const GraphArgs &g, const OpArgs &op,
                        const LaunchCfg &c, cudaStream_t s);
 cudaError_t launch_init(int gather, const OpArgs &op, int64_t rows, cudaStream_t s);

@@ -125,12 +125,6 @@ ug_status lower(const ug_graph *g, const ug_op_info *op, Lowered *out) {
 }
 
 // ------------------------------------------------------------------------- resolution
-// dot under SV runs the tile-major partial-dot kernel when the partials are additive (assign,
-// sum, mean) and no column tile straddles two heads.
-static bool split_dot_ok(const Lowered &lw, int vec) {
-    return lw.dot && lw.gather != UG_GATHER_MAX && lw.gather != UG_GATHER_MIN &&
-           (lw.args.H == 1 || lw.args.D % (32 * vec) == 0);
-}
 
 ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, LaunchCfg *cfg) {
     (void)g;
@@ -169,10 +163,7 @@ ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, La
         c.L = L;
     }
     if (c.strategy == UG_BE) c.L = std::min(32, need);
-    if (c.strategy == UG_SV && lw.dot) {
-        if (split_dot_ok(lw, c.vec)) { c.ftile = 32 * c.vec; c.L = 32; }
-        else c.G = 1;                              // one row per lane group (k_dot)
-    }
+    if (c.strategy == UG_SV && lw.dot) c.G = 1;   // dot under SV: one row per lane group (k_dot)
     *cfg = c;
     return UG_OK;
 }
@@ -236,7 +227,6 @@ static int launches_for(const Lowered &lw, const LaunchCfg &c, int64_t n_split_r
     if (lw.to_edges) return 1;
     if (edge_units) return lw.gather == UG_GATHER_SUM ? 2 : 3;
     if (c.strategy == UG_SV && !lw.dot) return n_split_rows > 0 ? 2 : 1;
-    if (c.strategy == UG_SV && split_dot_ok(lw, c.vec)) return lw.gather == UG_GATHER_MEAN ? 3 : 2;
     return 1;
 }
 
@@ -311,12 +301,6 @@ static ug_status run(const ug_graph *g, const ug_op_info *op, const ug_schedule 
             if (ev_end) cudaEventRecord(ev_end, s);
         }
         if (err == cudaSuccess && lw.gather != UG_GATHER_SUM) err = launch_epilogue(lw.gather, ga, lw.args, s);
-    } else if (lw.dot && c.strategy == UG_SV && split_dot_ok(lw, c.vec)) {
-        const SplitPlan *plan = nullptr;
-        if ((st = get_plan(g, c.G, &plan)) != UG_OK) return st;
-        err = launch_init(UG_GATHER_SUM, lw.args, lw.to_edges ? g->E : g->V, s);   // zero the output
-        if (err == cudaSuccess) err = launch_split_dot(lw.gather, ga, lw.args, c, *plan, s, ev_begin, ev_end);
-        if (err == cudaSuccess && lw.gather == UG_GATHER_MEAN) err = launch_epilogue(lw.gather, ga, lw.args, s);
     } else if (lw.dot) {
         if (ev_begin) cudaEventRecord(ev_begin, s);
         err = launch_dot(!edge_units, lw.gather, ga, lw.args, c, s);

@@ -33,16 +33,17 @@ def main():
     ap.add_argument("--F", type=int, default=64)
     ap.add_argument("--schedule", default=None)
     ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--ld", type=int, default=None, help="row stride of the feature tensor (padding)")
     a = ap.parse_args()
     c = ugdata.CONFIGS[a.config]
     src, dst = ugdata.graph(a.config)
     V, E = c.V, len(src)
     g = ug.Graph(V, src, dst)
     eo, go, at, bt, ct = OPS[a.op]
-    X = torch.rand(V, a.F, device="cuda") - 0.5
+    X = (torch.rand(V, a.ld or a.F, device="cuda") - 0.5)[:, :a.F]
     B = {"e": torch.rand(E, 1, device="cuda") + 0.5, "v": X, "u": X, None: None}[bt]
     W = 1 if eo == "dot" else a.F
-    C = torch.empty(V if ct == "v" else E, W, device="cuda")
+    C = torch.empty(V if ct == "v" else E, (a.ld or W) if W > 1 else 1, device="cuda")[:, :W]
     kw = dict(A=X, a_type=at, B=B, b_type=bt, C=C, c_type=ct, F=a.F, H=1)
     sched = a.schedule or ug.schedule_select(g, eo, go, **kw)
     ts = []
@@ -54,7 +55,7 @@ def main():
         e1.record()
         torch.cuda.synchronize()
         ts.append(e0.elapsed_time(e1))
-    print(f"{a.config} {a.op} F={a.F} {sched}: median {statistics.median(ts) * 1e3:.1f} us")
+    print(f"{a.config} {a.op} F={a.F} ld={a.ld or a.F} {sched}: median {statistics.median(ts) * 1e3:.1f} us")
 
 
 if __name__ == "__main__":
