@@ -103,7 +103,12 @@ typedef struct {
     int32_t block_threads;  /* CTA size (0 -> 256)                                              */
     int32_t ftile;          /* column-tile width for L2 blocking, tile-major grid order; 0 = off */
     int32_t vec;            /* feature vector width 1/2/4; 0 -> widest the layout allows        */
+    int32_t flags;          /* UG_SCHED_PACK (SV only): first stage a full-width Src_V operand whose
+                               rows are not 128-byte aligned into an aligned scratch copy, so each
+                               column slab occupies whole L2 lines and rows take 16-byte loads   */
 } ug_schedule;
+
+#define UG_SCHED_PACK 1
 
 /* Optional allocator for graph-owned device arrays (e.g. torch's caching allocator).
  * NULL -> cudaMallocAsync / cudaFreeAsync on the given stream. */

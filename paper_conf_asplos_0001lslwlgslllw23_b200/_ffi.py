@@ -38,7 +38,8 @@ class UgOpInfo(ctypes.Structure):
 
 class UgSchedule(ctypes.Structure):
     _fields_ = [("strategy", ctypes.c_int32), ("group", ctypes.c_int32), ("tile", ctypes.c_int32),
-                ("block_threads", ctypes.c_int32), ("ftile", ctypes.c_int32), ("vec", ctypes.c_int32)]
+                ("block_threads", ctypes.c_int32), ("ftile", ctypes.c_int32), ("vec", ctypes.c_int32),
+                ("flags", ctypes.c_int32)]
 
 
 class UgAllocator(ctypes.Structure):

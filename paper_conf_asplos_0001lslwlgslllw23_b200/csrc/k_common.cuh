@@ -171,6 +171,22 @@ __device__ __forceinline__ void st_vec_n(float *p, const float (&r)[VEC], int n)
         if (i < n) p[i] = r[i];
 }
 
+// Store n (<= VEC) values into C whose rows only guarantee `cvec`-wide alignment (SV loads
+// with a wider vector than C's layout allows: e.g. float4 loads, 8-byte-aligned output rows).
+template <int VEC>
+__device__ __forceinline__ void st_out(float *p, const float (&r)[VEC], int n, int cvec) {
+    if (n >= VEC && cvec >= VEC) {
+        st_vec<VEC>(p, r);
+    } else if (VEC == 4 && n >= 4 && cvec >= 2) {
+        *reinterpret_cast<float2 *>(p) = make_float2(r[0], r[1]);
+        *reinterpret_cast<float2 *>(p + 2) = make_float2(r[VEC > 2 ? 2 : 0], r[VEC > 3 ? 3 : 0]);
+    } else {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i)
+            if (i < n) p[i] = r[i];
+    }
+}
+
 // Row of an operand for the edge (src, dst, e): type_idx_dict.
 __device__ __forceinline__ int64_t op_row(int32_t type, int64_t src, int64_t dst, int64_t e) {
     return type == UG_T_SRC_V ? src : (type == UG_T_DST_V ? dst : e);

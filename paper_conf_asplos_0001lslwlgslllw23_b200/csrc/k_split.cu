@@ -95,7 +95,7 @@ __global__ void __launch_bounds__(256) k_split(GraphArgs g, OpArgs op, const int
             const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
             float m[VEC];
             message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m);
-            st_vec_n<VEC>(op.C + e * op.c_ld + f, m, op.W - f);
+            st_out<VEC>(op.C + e * op.c_ld + f, m, op.W - f, op.c_vec);
         }
     } else {
         float acc[VEC];
@@ -144,8 +144,8 @@ __global__ void __launch_bounds__(256) k_split(GraphArgs g, OpArgs op, const int
             float out[VEC];
 #pragma unroll
             for (int i = 0; i < VEC; ++i) out[i] = g_finalize<GOP>(acc[i], deg);
-            if (f + VEC <= op.W) st_vec_hint<VEC>(op.C + v * op.c_ld + f, out, wpol);
-            else st_vec_n<VEC>(op.C + v * op.c_ld + f, out, op.W - f);
+            if (f + VEC <= op.W && op.c_vec >= VEC) st_vec_hint<VEC>(op.C + v * op.c_ld + f, out, wpol);
+            else st_out<VEC>(op.C + v * op.c_ld + f, out, op.W - f, op.c_vec);
         } else {
             st_vec_hint<VEC>(scratch + (int64_t)ch.w * sld + f, acc, wpol);
         }
@@ -175,7 +175,7 @@ __global__ void k_split_fix(GraphArgs g, OpArgs op, const int4 *__restrict__ spl
     const int64_t deg = (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
 #pragma unroll
     for (int i = 0; i < VEC; ++i) acc[i] = g_finalize<GOP>(acc[i], deg);
-    st_vec_n<VEC>(op.C + v * op.c_ld + f, acc, op.W - f);
+    st_out<VEC>(op.C + v * op.c_ld + f, acc, op.W - f, op.c_vec);
 }
 
 cudaError_t launch_split_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,

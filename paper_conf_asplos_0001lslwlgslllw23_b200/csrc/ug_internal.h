@@ -41,6 +41,7 @@ struct OpArgs {
     int32_t F;        // feature width
     int32_t W;        // message / output width (F, or H for dot)
     int32_t H, D;     // heads, D = F / H
+    int32_t c_vec;    // widest aligned vector store into C (may be < the load width under SV)
 };
 
 // Normalised edge ops inside the kernels (copy_rhs is rewritten as copy_lhs on B).
@@ -53,6 +54,7 @@ struct LaunchCfg {
     int block;        // CTA size
     int ftile;        // column tile width (multiple of vec), 0 = whole width
     int vec;          // 1, 2, 4
+    bool pack;        // UG_SCHED_PACK: stage A into 128-byte-aligned rows first (SV only)
 };
 
 // Split-row plan for UG_SV (built once per (graph, chunk size), cached on the graph).

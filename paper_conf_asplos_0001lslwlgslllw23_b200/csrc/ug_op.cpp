@@ -98,28 +98,30 @@ ug_status lower(const ug_graph *g, const ug_op_info *op, Lowered *out) {
     if (lw.op_class == 1 && (go == UG_GATHER_MAX || go == UG_GATHER_MIN)) lw.op_class = 5;
     else if (lw.op_class == 1 && opb) lw.op_class = 4;
 
-    // Widest legal feature vector (R22 in DESIGN.md): every full-width operand row must be
-    // aligned and either F % vec == 0 or padded (ld >= round_up(F, vec)); a broadcast operand
-    // must keep a vec chunk inside one head; C stores must be aligned.
-    lw.max_vec = 1;
-    for (int v : {4, 2}) {
-        bool ok = true;
-        const int span = dot ? lw.args.D : F;
-        for (int i = 0; i < 2 && ok; ++i) {
-            const ug_tensor *t = used[i];
-            if (!t) continue;
-            const Operand &o = *dst_ops[i];
-            if (o.div == 1) {
-                ok = (o.ld % v == 0) && ((uintptr_t)o.p % (4 * v) == 0) &&
-                     (span % v == 0 || o.ld >= ((F + v - 1) / v) * v);
-            } else {
-                ok = (o.div % v == 0);
-            }
+    // Widest legal feature vector (R22 in DESIGN.md), per tensor: a full-width operand row must
+    // be aligned and either F % vec == 0 or padded (ld >= round_up(F, vec)); a broadcast operand
+    // must keep a vec chunk inside one head; C stores must be aligned (dot: D % vec == 0).
+    const int span = dot ? lw.args.D : F;
+    auto operand_vec = [&](const ug_tensor *t, const Operand &o) {
+        if (!t) return 4;
+        for (int v : {4, 2}) {
+            const bool ok = o.div == 1 ? (o.ld % v == 0) && ((uintptr_t)o.p % (4 * v) == 0) &&
+                                             (span % v == 0 || o.ld >= ((F + v - 1) / v) * v)
+                                       : (o.div % v == 0);
+            if (ok) return v;
         }
-        if (ok && !dot) ok = (C.ld % v == 0) && ((uintptr_t)C.data % (4 * v) == 0);
-        if (ok && dot) ok = (lw.args.D % v == 0);
-        if (ok) { lw.max_vec = v; break; }
+        return 1;
+    };
+    lw.a_vec = operand_vec(opa, oa);
+    lw.b_vec = operand_vec(opb, ob);
+    lw.c_vec = 1;
+    for (int v : {4, 2}) {
+        const bool ok = dot ? (lw.args.D % v == 0) : (C.ld % v == 0) && ((uintptr_t)C.data % (4 * v) == 0);
+        if (ok) { lw.c_vec = v; break; }
     }
+    lw.max_vec = std::min(std::min(lw.a_vec, lw.b_vec), lw.c_vec);
+    lw.args.c_vec = dot ? 1 : lw.c_vec;
+    lw.pack_ok = !dot && opa && oa.type == UG_T_SRC_V && oa.div == 1 && (oa.ld * 4) % 128 != 0;
     *out = lw;
     return UG_OK;
 }
@@ -132,9 +134,14 @@ ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, La
     c.strategy = s.strategy;
     if (c.strategy < UG_TV || c.strategy > UG_SV)
         return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "strategy out of range");
-    c.vec = s.vec ? s.vec : lw.max_vec;
+    // SV stores through any C alignment (st_out), so its vector width is bounded by the operands
+    // only; with UG_SCHED_PACK the staged copy of A is 16-byte aligned (a_vec = 4).
+    c.pack = c.strategy == UG_SV && (s.flags & UG_SCHED_PACK) && lw.pack_ok;
+    const int sv_vec = std::min(c.pack ? 4 : lw.a_vec, lw.b_vec);
+    const int allowed = (c.strategy == UG_SV && !lw.dot) ? sv_vec : lw.max_vec;
+    c.vec = s.vec ? s.vec : allowed;
     if (!(c.vec == 1 || c.vec == 2 || c.vec == 4)) return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "vec must be 1, 2 or 4");
-    if (c.vec > lw.max_vec) return set_error(UG_ERR_ALIGNMENT, "forced vec wider than the operand layout allows");
+    if (c.vec > allowed) return set_error(UG_ERR_ALIGNMENT, "forced vec wider than the operand layout allows");
     c.G = s.group > 0 ? s.group : (c.strategy == UG_SV ? 2048 : 1);
     const int T = s.tile > 0 ? s.tile : 1;
     if (!is_pow2(T)) return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "tile T must be a power of two");
@@ -320,15 +327,29 @@ static ug_status run(const ug_graph *g, const ug_op_info *op, const ug_schedule 
     } else {  // UG_SV
         const SplitPlan *plan = nullptr;
         if ((st = get_plan(g, c.G, &plan)) != UG_OK) return st;
-        float *scratch = nullptr;
+        float *scratch = nullptr, *packed = nullptr;
         const int64_t sld = (lw.args.W + 3) / 4 * 4;
+        OpArgs args = lw.args;
+        if (c.pack) {
+            // stage A into rows of round_up(F, 32) floats (128-byte aligned): one 2-D copy
+            ensure_pool_retains();
+            const int64_t ldp = (int64_t)(lw.args.F + 31) / 32 * 32;
+            err = cudaMallocAsync((void **)&packed, sizeof(float) * (size_t)(g->V_total * ldp), s);
+            if (err != cudaSuccess) return set_error(UG_ERR_OOM, "SV pack allocation failed");
+            err = cudaMemcpy2DAsync(packed, sizeof(float) * ldp, args.A.p, sizeof(float) * args.A.ld,
+                                    sizeof(float) * lw.args.F, (size_t)g->V_total, cudaMemcpyDeviceToDevice, s);
+            if (err != cudaSuccess) { cudaFreeAsync(packed, s); return set_error(UG_ERR_CUDA, "SV pack copy failed"); }
+            args.A.p = packed;
+            args.A.ld = ldp;
+        }
         if (agg && plan->n_split_chunks > 0) {
             ensure_pool_retains();
             err = cudaMallocAsync((void **)&scratch, sizeof(float) * (size_t)(plan->n_split_chunks * sld), s);
             if (err != cudaSuccess) return set_error(UG_ERR_OOM, "SV scratch allocation failed");
         }
-        err = launch_split_vertex(lw.kedge, lw.gather, ga, lw.args, c, *plan, scratch, s, ev_begin, ev_end);
+        err = launch_split_vertex(lw.kedge, lw.gather, ga, args, c, *plan, scratch, s, ev_begin, ev_end);
         if (scratch) cudaFreeAsync(scratch, s);
+        if (packed) cudaFreeAsync(packed, s);
     }
     if (err != cudaSuccess) return set_error(UG_ERR_CUDA, std::string("kernel launch: ") + cudaGetErrorString(err));
     return UG_OK;
@@ -378,6 +399,7 @@ extern "C" ug_status ug_schedule_parse(const char *text, ug_schedule *out) {
         case 'B': s.block_threads = (int32_t)val; break;
         case 'F': s.ftile = (int32_t)val; break;
         case 'V': s.vec = (int32_t)val; break;
+        case 'P': s.flags = val ? (s.flags | UG_SCHED_PACK) : (s.flags & ~UG_SCHED_PACK); break;
         default: return set_error(UG_ERR_INVALID_ARG, "bad schedule token '" + tok + "'");
         }
         pos = nxt;
@@ -396,6 +418,7 @@ extern "C" ug_status ug_schedule_format(const ug_schedule *s, char *buf, size_t 
         if (s->ftile) r += "_F" + std::to_string(s->ftile);
         if (s->block_threads) r += "_B" + std::to_string(s->block_threads);
         if (s->vec) r += "_V" + std::to_string(s->vec);
+        if (s->flags & UG_SCHED_PACK) r += "_P1";
     }
     std::snprintf(buf, len, "%s", r.c_str());
     return UG_OK;

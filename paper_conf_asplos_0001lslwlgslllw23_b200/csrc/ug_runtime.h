@@ -17,7 +17,9 @@ struct Lowered {
     int gather;         // UG_GATHER_*
     bool to_edges;      // C is an Edge tensor (message creation)
     OpArgs args;
-    int max_vec;        // widest legal feature vector (1, 2, 4)
+    int max_vec;        // widest legal feature vector for every tensor (1, 2, 4)
+    int a_vec, b_vec, c_vec;   // per tensor
+    bool pack_ok;       // A is a full-width Src_V operand whose rows are not 128-byte aligned
     // selector key
     int op_class;       // 0 msg, 1 agg (copy, sum/mean), 2 dot msg, 3 dot agg, 4 agg_bin, 5 agg_ext
 };

@@ -19,7 +19,7 @@ ug = pytest.importorskip("paper_conf_asplos_0001lslwlgslllw23_b200")
 # with grouping / tiling / tile-major variants.  Each is exercised on all 160 ops.
 SCHEDULES = ["TV_G1_T1", "TV_G3_T4", "WV_G1_T1", "WV_G2_T2_F8", "TE_G1_T4", "TE_G5_T32",
              "WE_G7_T1", "WE_G2_T2_F8", "BV_G1", "BV_G3_B128", "BE_G64", "SV_G7", "SV_G64_F8",
-             "TV_G1_T8_V1", "WE_G4_T1_V1"]
+             "TV_G1_T8_V1", "WE_G4_T1_V1", "SV_G16_P1", "SV_G64_F8_P1"]
 
 
 @pytest.fixture(scope="module")
@@ -59,7 +59,7 @@ def test_auto_schedule_and_broadcast_vertex(small_graph, op):
 
 
 @pytest.mark.parametrize("layout", [(None, 0), (24, 0), (23, 1), (20, 2)])
-@pytest.mark.parametrize("sch", ["WV_G1_T1", "TE_G2_T8", "SV_G16", "BV_G1", "TV_G1_T4", None])
+@pytest.mark.parametrize("sch", ["WV_G1_T1", "TE_G2_T8", "SV_G16", "SV_G16_P1", "BV_G1", "TV_G1_T4", None])
 def test_strided_and_misaligned_layouts(small_graph, layout, sch):
     """Row stride ld > width and 4/8-byte-offset base pointers select narrower vectors."""
     V, E, src, dst, g = small_graph
