@@ -307,7 +307,22 @@ def main():
         e.record(stream)   # materialise the cudaEvent_t handles
     torch.cuda.synchronize()
 
+    # N > 1, single-operand aggregation (copy_u_*): column-chunked all-gather overlapped with
+    # the per-chunk op (ShardedOperator.run_chunked); otherwise gather X, then one op.
+    chunked = world > 1 and b_t is None and go != "assign"
+    bufs = sh.chunk_buffers(F, 64, dev) if chunked else None
+    if chunked:
+        launches = sum(ug.launch_count(g, eo, go, A=bufs["full"][c][:V], a_type="u", C=Y[:, c0:c1], c_type="v",
+                                       F=c1 - c0, H=1) for c, (c0, c1) in enumerate(bufs["cols"]))
+
     def step(i=None):
+        if chunked:
+            if i is not None:
+                ev_k0[i].record(stream)
+            sh.run_chunked(eo, go, X_local, Y, chunk=64, buffers=bufs)
+            if i is not None:
+                ev_k1[i].record(stream)
+            return
         if world > 1:
             sh.gather_x(X_local, X_full)          # the exchange: NCCL all-gather of X row blocks
         if i is None:
@@ -375,8 +390,11 @@ def main():
             e0.record(stream)
             for i in range(n_e2e):
                 Xl.copy_(Xlh, non_blocking=True)
-                sh.gather_x(Xl, X_full)
-                ug.op_run(g, eo, go, schedule=chosen, **kw)
+                if chunked:
+                    sh.run_chunked(eo, go, Xl, Y, chunk=64, buffers=bufs)
+                else:
+                    sh.gather_x(Xl, X_full)
+                    ug.op_run(g, eo, go, schedule=chosen, **kw)
                 Yh[i % 2].copy_(Y, non_blocking=True)
             e1.record(stream)
             torch.cuda.synchronize()
@@ -420,13 +438,16 @@ def main():
                        "schedule": chosen, "graph": "Chung-Lu lognormal degrees (ugdata), seed %d" % cfg.seed,
                        "l2": "inputs larger than L2 (X %.0f MB, col_idx %.0f MB > 126 MB): no flush"
                              % (V * F * 4 / 1e6, E * 4 / 1e6),
-                       "parallelism": f"dst-row sharding x{world}" + (" + NCCL all-gather of X" if world > 1 else ""),
+                       "parallelism": f"dst-row sharding x{world}" + (
+                           (" + column-chunked NCCL all-gather of X overlapped with the op" if chunked
+                            else " + NCCL all-gather of X") if world > 1 else ""),
                        "logical_bytes": by},
             "latency_ms": round(ms, 4),
             "frac_of_8TBps": round(value / 8000.0, 4),
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": traffic,
-                         "kernel": "k_split (SV main traversal)" if chosen.startswith("SV") else "main traversal",
+                         "kernel": ("k_split per 64-column chunk, exchange overlapped" if chunked else
+                                    "k_split (SV main traversal)" if chosen.startswith("SV") else "main traversal"),
                          "kernel_ms": round(kms, 4), "peak_source": peak_src,
                          "bytes": "algorithmic (SURVEY 8(d)) per launch, this rank's rows"},
             "cpu_baseline": cpu,

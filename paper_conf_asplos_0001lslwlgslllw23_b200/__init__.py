@@ -120,6 +120,12 @@ class Graph:
         check(lib.ug_graph_csr(self._h, rp.ctypes.data, col.ctypes.data, eid.ctypes.data), "ug_graph_csr")
         return rp, col[:s["E"]], eid[:s["E"]]
 
+    def row_ptr(self):
+        """Host row_ptr[V+1] only (local positions for a view)."""
+        rp = np.zeros(self.stats()["V"] + 1, np.int32)
+        check(lib.ug_graph_csr(self._h, rp.ctypes.data, None, None), "ug_graph_csr")
+        return rp
+
     def partition(self, parts):
         out = np.zeros(parts + 1, np.int64)
         check(lib.ug_graph_partition(self._h, int(parts), out.ctypes.data), "ug_graph_partition")

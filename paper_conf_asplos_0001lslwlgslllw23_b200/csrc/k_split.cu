@@ -19,8 +19,9 @@
 namespace ug {
 
 // Inner in-edge loop of the SV fast path.  BM: 0 no B operand, 1 B is Dst_V (constant over
-// the row: loaded once), 2 B is an Edge tensor (row = CSR position), 3 B is Src_V.  All offsets
-// are 32-bit (the host checks rows * ld < 2^32).  Advances k to the last multiple of 8.
+// the row: loaded once), 2 / 3 B is an Edge tensor (row = CSR position) with per-head broadcast
+// / full width, 4 / 5 B is Src_V with broadcast / full width.  All offsets are 32-bit (the
+// host checks rows * ld < 2^32).  Advances k to the last multiple of UF.
 template <int KE, int GOP, int VEC, int BM>
 __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t &k,
                                                 int64_t k1, int f, int64_t cb, float (&acc)[VEC]) {
@@ -31,7 +32,7 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
     const uint64_t stream = l2_policy_evict_first();  // col_idx / edge tensors: read once per pass
     const uint32_t lda = (uint32_t)op.A.ld, fo = (uint32_t)f;
     const uint32_t ldb = (uint32_t)op.B.ld, cbo = (uint32_t)cb;
-    const bool bfull = op.B.div == 1;
+    constexpr bool bfull = BM == 3 || BM == 5;
     float bconst[VEC];
     if constexpr (BM == 1) fetch<VEC>(op.B, v, cb, bconst);
     for (; k + UF <= k1; k += UF) {
@@ -49,10 +50,10 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
 #pragma unroll
                     for (int i = 0; i < VEC; ++i) b[i] = bconst[i];
                 } else {
-                    const uint32_t row = BM == 2 ? (uint32_t)(k + q) : s[q];
+                    const uint32_t row = (BM == 2 || BM == 3) ? (uint32_t)(k + q) : s[q];
                     const float *bp = op.B.p + (row * ldb + cbo);
-                    if (bfull) {
-                        ldg_vec_hint<VEC>(bp, b, BM == 2 ? stream : keep);
+                    if constexpr (bfull) {
+                        ldg_vec_hint<VEC>(bp, b, BM == 3 ? stream : keep);
                     } else {
                         const float x = __ldg(bp);
 #pragma unroll
@@ -107,12 +108,19 @@ __global__ void __launch_bounds__(256) k_split(GraphArgs g, OpArgs op, const int
             // the row address is one IMAD + IMAD.WIDE from the (warp-uniform, L1-broadcast)
             // column index, so each in-edge costs ~6 instructions per lane.  The B operand's
             // addressing mode is resolved once per unit (a Dst_V operand is loaded once).
-            const int bm = KE == K_COPY ? 0 : (op.B.type == UG_T_DST_V ? 1 : (op.B.type == UG_T_EDGE ? 2 : 3));
-            switch (bm) {
-            case 0: split_fast_loop<KE, GOP, VEC, 0>(g, op, v, k, k1, f, cb, acc); break;
-            case 1: split_fast_loop<KE, GOP, VEC, 1>(g, op, v, k, k1, f, cb, acc); break;
-            case 2: split_fast_loop<KE, GOP, VEC, 2>(g, op, v, k, k1, f, cb, acc); break;
-            default: split_fast_loop<KE, GOP, VEC, 3>(g, op, v, k, k1, f, cb, acc); break;
+            const int bfl = op.B.div == 1 ? 1 : 0;
+            const int bm = KE == K_COPY ? 0
+                         : op.B.type == UG_T_DST_V ? 1 : (op.B.type == UG_T_EDGE ? 2 + bfl : 4 + bfl);
+            if constexpr (KE == K_COPY) {
+                split_fast_loop<KE, GOP, VEC, 0>(g, op, v, k, k1, f, cb, acc);
+            } else {
+                switch (bm) {
+                case 1: split_fast_loop<KE, GOP, VEC, 1>(g, op, v, k, k1, f, cb, acc); break;
+                case 2: split_fast_loop<KE, GOP, VEC, 2>(g, op, v, k, k1, f, cb, acc); break;
+                case 3: split_fast_loop<KE, GOP, VEC, 3>(g, op, v, k, k1, f, cb, acc); break;
+                case 4: split_fast_loop<KE, GOP, VEC, 4>(g, op, v, k, k1, f, cb, acc); break;
+                default: split_fast_loop<KE, GOP, VEC, 5>(g, op, v, k, k1, f, cb, acc); break;
+                }
             }
         } else {
             for (; k + U <= k1; k += U) {

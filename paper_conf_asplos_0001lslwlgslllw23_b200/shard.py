@@ -43,7 +43,7 @@ class ShardedOperator:
         self.splits = graph.partition(world)
         self.r0, self.r1 = int(self.splits[rank]), int(self.splits[rank + 1])
         self.view = graph.view_rows(self.r0, self.r1) if world > 1 else graph
-        rp = graph.csr()[0]
+        rp = graph.row_ptr()
         self.e0, self.e1 = int(rp[self.r0]), int(rp[self.r1])
         self.blk = block_rows(self.V, world)
 
@@ -77,6 +77,40 @@ class ShardedOperator:
         op_run(self.view, edge_op, gather_op, A=X_full[: self.V], a_type="u", B=B, b_type=b_type, C=C_local,
                c_type="v", F=F, H=H, schedule=schedule)
         return C_local
+
+    def run_chunked(self, edge_op, gather_op, X_local, C_local, chunk=64, schedule=None, buffers=None):
+        """Sharded step with the exchange overlapped (SURVEY 8(e) overlap option): X is
+        all-gathered in column chunks (the paper's feature-tiling axis) on a side
+        stream while the operator runs on the previous chunk; every chunk's op writes its own
+        columns of C_local.  Only ops whose sole feature operand is the Src_V X (copy_u_*) are
+        column-separable this way.  `buffers` (from chunk_buffers) are reused across steps."""
+        import torch.distributed as dist
+        from . import op_run
+        F = X_local.shape[1]
+        bufs = buffers or self.chunk_buffers(F, chunk, X_local.device)
+        main = torch.cuda.current_stream(X_local.device)
+        side = bufs["stream"]
+        side.wait_stream(main)                       # X_local is ready
+        for c, (c0, c1) in enumerate(bufs["cols"]):
+            with torch.cuda.stream(side):
+                bufs["send"][c].copy_(X_local[:, c0:c1])
+                if self.world == 1:
+                    bufs["full"][c].copy_(bufs["send"][c])
+                else:
+                    dist.all_gather_into_tensor(bufs["full"][c], bufs["send"][c], group=self.group)
+                bufs["ready"][c].record(side)
+        for c, (c0, c1) in enumerate(bufs["cols"]):
+            main.wait_event(bufs["ready"][c])
+            op_run(self.view, edge_op, gather_op, A=bufs["full"][c][: self.V], a_type="u",
+                   C=C_local[:, c0:c1], c_type="v", F=c1 - c0, H=1, schedule=schedule)
+        return C_local
+
+    def chunk_buffers(self, F, chunk, device):
+        cols = [(c0, min(F, c0 + chunk)) for c0 in range(0, F, chunk)]
+        return {"cols": cols, "stream": torch.cuda.Stream(device),
+                "send": [torch.empty(self.blk, c1 - c0, device=device) for c0, c1 in cols],
+                "full": [torch.empty(self.blk * self.world, c1 - c0, device=device) for c0, c1 in cols],
+                "ready": [torch.cuda.Event() for _ in cols]}
 
     def gather_rows(self, Y_local: torch.Tensor) -> torch.Tensor:
         """Reassemble the row-sharded output on every rank (verification / next-layer input)."""

@@ -170,7 +170,7 @@ def test_validate_rejects_width_mismatch():
 
 
 @pytest.mark.parametrize("text", ["TE_G1_T16", "WV_G4_T2", "TV_G1_T1", "WE_G64_T1", "BV_G2",
-                                  "BE_G256", "SV_G2048_F64", "SV_G1024_F128_B128_V4"])
+                                  "BE_G256", "SV_G2048_F64", "SV_G1024_F128_B128_V4", "SV_G512_F64_P1"])
 def test_schedule_text_roundtrip(text):
     s = ug.parse_schedule(text)
     assert ug.parse_schedule(ug.format_schedule(s)).strategy == s.strategy

@@ -130,3 +130,17 @@ def test_prepared_op_and_cuda_graph_capture():
               schedule=chain[-1].schedule)
     torch.cuda.synchronize()
     torch.testing.assert_close(Y2, ref, rtol=1e-5, atol=1e-5)
+
+
+def test_sharded_chunked_world1_matches_op_run(c3):
+    """run_chunked (column-chunked exchange overlapped with the op) == one op_run, per column."""
+    V, src, dst, g = c3
+    sh = ShardedOperator(g, 1, 0)
+    X = torch.from_numpy(ugdata.values(V, 150, 4, 1, mode="int")).cuda()
+    for gop in ("sum", "mean", "max"):
+        Y = torch.empty(V, 150, device="cuda")
+        sh.run_chunked("copy_lhs", gop, x_block(X, V, 1, 0), Y, chunk=64)
+        Y2 = torch.empty(V, 150, device="cuda")
+        ug.op_run(g, "copy_lhs", gop, A=X, a_type="u", C=Y2, c_type="v")
+        torch.cuda.synchronize()
+        assert torch.equal(Y, Y2), gop
