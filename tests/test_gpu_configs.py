@@ -180,3 +180,26 @@ def view_row_base(g, r0, r1):
         _rp_cache[key] = g.csr()[0]
     rp = _rp_cache[key]
     return int(rp[r0]), int(rp[r1])
+
+
+@pytest.mark.parametrize("cfg, op, sch", [
+    ("C5", ("copy_lhs", "u", None, "sum", "v"), None),
+    ("C5", ("copy_lhs", "u", None, "mean", "v"), "SV_G2048_F128_P1"),
+    ("C3", ("mul", "u", "e", "sum", "v"), None),
+    ("C3", ("mul", "u", "e", "sum", "v"), "TE_G32_T16"),
+])
+def test_positive_stress_accumulation(cfg, op, sch):
+    """All-positive inputs (partial sums grow linearly, the worst case for fp32 accumulation,
+    SURVEY 7 hard part 4): still within 1e-5 * sum|terms| on the hub rows and the sample."""
+    d = config_graph(cfg)
+    eo, l, r, gop, c = op
+    F = SHAPES[cfg]["F"]
+    A = ugdata.values(d["V"], F, 77, 1, mode="pos")
+    B = ugdata.values(d["E"], 1, 77, 2, mode="pos") if r == "e" else None
+    C = out_tensor(op, d["V"], d["E"], F, 1)
+    ug.op_run(d["g"], eo, gop, A=to_dev(A), a_type=l, B=to_dev(B), b_type=r, C=C, c_type=c, F=F, H=1,
+              schedule=sch)
+    torch.cuda.synchronize()
+    (ref, bnd), rows = sampled_oracle(op, d, A, B, F, 1, False)
+    got = C[torch.from_numpy(rows).cuda()].cpu().numpy()
+    assert_parity(op, got, ref, bnd, False, what=f"{cfg} {op} {sch} positive-stress")
