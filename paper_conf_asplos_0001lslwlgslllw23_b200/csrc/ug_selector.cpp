@@ -9,6 +9,7 @@
 // over a few hundred entries: well under the paper's 0.2 ms budget.
 #include <dlfcn.h>
 
+#include <algorithm>
 #include <cctype>
 #include <cstdlib>
 #include <cstring>
@@ -142,7 +143,10 @@ static ug_schedule prior(const ug_graph *g, const Lowered &lw) {
     } else if (lw.op_class == 3) {
         s.strategy = UG_WV; s.group = 1; s.tile = 1;
     } else {                           // aggregation (classes 1, 4, 5)
-        if (W >= 32 || g->max_deg > 256) { s.strategy = UG_SV; s.group = 1024; s.ftile = 0; }
+        if (W >= 32 || g->max_deg > 256) {
+            s.strategy = UG_SV; s.group = 512; s.ftile = 0;
+            if (W >= 256 && lw.pack_ok) s.flags = UG_SCHED_PACK;   // wide rows: aligned L2 slabs
+        }
         else { s.strategy = UG_WV; s.group = 1; s.tile = 1; }
     }
     return s;
@@ -169,6 +173,13 @@ ug_status select_schedule(const ug_graph *g, const Lowered &lw, ug_schedule *out
                 continue;
             ug_schedule s = e.sched;
             if (s.vec > lw.max_vec) s.vec = 0;   // table entry measured on an aligned layout
+            if (s.strategy == UG_SV && s.ftile > 0) {
+                // the entry's column tile may need more than 32 lanes at this layout's vector
+                // width (measured with float4 rows, applied to float2 rows): keep 32 lanes
+                const bool pack = (s.flags & UG_SCHED_PACK) && lw.pack_ok;
+                const int vec = std::max(1, std::min(pack ? 4 : lw.a_vec, lw.b_vec));
+                if (s.ftile / vec > 32 || s.ftile % vec) s.ftile = 32 * vec;
+            }
             *out = s;
             return UG_OK;
         }
