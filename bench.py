@@ -231,7 +231,55 @@ def secondary_configs(ug, torch, dev, reps=20, warm=5):
                     "host_launch_prepared_us": round(prep_us, 2)})
         del A, B, C
     del scrub
+    out.append(gat_chain_graph(ug, torch, dev, graphs["C2"][0]))
     return out
+
+
+def gat_chain_graph(ug, torch, dev, g, reps=50):
+    """C2 GAT attention chain (u_add_v -> e_max -> e_div_v -> e_sum -> e_div_v -> u_mul_e_sum,
+    6 graph ops) issued eagerly through PreparedOp vs replayed as one CUDA graph:
+    small graphs are launch-bound, a captured chain removes the host cost per op."""
+    import ugdata
+    c = ugdata.CONFIGS["C2"]
+    V, E, H, F = c.V, c.E, 8, 64
+    X = torch.rand(V, F, device=dev)
+    el, er = torch.rand(V, H, device=dev) + 0.5, torch.rand(V, H, device=dev) + 0.5
+    a, s, p = (torch.empty(E, H, device=dev) for _ in range(3))
+    m, den = torch.empty(V, H, device=dev), torch.empty(V, H, device=dev)
+    Y = torch.empty(V, F, device=dev)
+    chain = [ug.prepare(g, "add", "assign", A=el, a_type="u", B=er, b_type="v", C=a, c_type="e", F=H, H=H),
+             ug.prepare(g, "copy_lhs", "max", A=a, a_type="e", C=m, c_type="v", F=H, H=H),
+             ug.prepare(g, "div", "assign", A=a, a_type="e", B=m, b_type="v", C=s, c_type="e", F=H, H=H),
+             ug.prepare(g, "copy_lhs", "sum", A=s, a_type="e", C=den, c_type="v", F=H, H=H),
+             ug.prepare(g, "div", "assign", A=s, a_type="e", B=den, b_type="v", C=p, c_type="e", F=H, H=H),
+             ug.prepare(g, "mul", "sum", A=X, a_type="u", B=p, b_type="e", C=Y, c_type="v", F=F, H=H)]
+    side = torch.cuda.Stream(dev)
+    with torch.cuda.stream(side):
+        for op in chain:
+            op()
+    torch.cuda.synchronize()
+    cg = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(cg):
+        for op in chain:
+            op()
+    torch.cuda.synchronize()
+
+    def timed(fn):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        fn()
+        torch.cuda.synchronize()
+        e0.record()
+        for _ in range(reps):
+            fn()
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / reps * 1e3
+
+    eager = timed(lambda: [op() for op in chain])
+    graph = timed(cg.replay)
+    return {"config": "C2", "op": "GAT attention chain (6 ops)", "F": F, "H": H,
+            "schedules": [op.schedule for op in chain],
+            "eager_us_per_chain": round(eager, 2), "cuda_graph_us_per_chain": round(graph, 2)}
 
 
 # ---------------------------------------------------------------------------- GPU run
@@ -267,12 +315,22 @@ def main():
     from paper_conf_asplos_0001lslwlgslllw23_b200.shard import ShardedOperator, x_block
 
     dist = None
+    # one process per GPU over NCCL; UG_DIST_BACKEND=gloo is a single-GPU dry run of the N > 1
+    # path (ranks share cuda:0, the exchange is staged through host memory) -- never a bench number
+    backend = os.environ.get("UG_DIST_BACKEND", "nccl")
+    dev = torch.device("cuda", local % max(1, torch.cuda.device_count()))
+    torch.cuda.set_device(dev)
     if world > 1:
         import torch.distributed as dist
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
-    torch.cuda.set_device(dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
+
+    def max_over_ranks(vals):
+        t = torch.tensor(vals, dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return [float(x) for x in t]
 
     src, dst = ugdata.graph(args.config)
     V, E = cfg.V, len(src)
@@ -336,7 +394,7 @@ def main():
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    with ClockSampler(local) as clocks:
+    with ClockSampler(dev.index) as clocks:
         for i in range(args.steps):
             ev_s0[i].record(stream)
             step(i)
@@ -348,9 +406,7 @@ def main():
     tot = sum(ev_s0[i].elapsed_time(ev_s1[i]) for i in range(args.steps))
     ktot = sum(ev_k0[i].elapsed_time(ev_k1[i]) for i in range(args.steps))
     if world > 1:
-        t = torch.tensor([tot, ktot], device=dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        tot, ktot = float(t[0]), float(t[1])
+        tot, ktot = max_over_ranks([tot, ktot])
     ms = tot / args.steps
     kms = ktot / args.steps
     by = logical_bytes(V, E, F, args.op)
@@ -398,9 +454,7 @@ def main():
                 Yh[i % 2].copy_(Y, non_blocking=True)
             e1.record(stream)
             torch.cuda.synchronize()
-            t = torch.tensor([e0.elapsed_time(e1) / n_e2e], device=dev, dtype=torch.float64)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            e_ms = float(t[0])
+            e_ms = max_over_ranks([e0.elapsed_time(e1) / n_e2e])[0]
         e2e = {"value": round(by / (e_ms * 1e-3) / 1e9, 1), "unit": "GB/s", "ms_per_step": round(e_ms, 3),
                "h2d_bytes_per_step": int((V if world == 1 else sh.blk * world) * F * 4),
                "d2h_bytes_per_step": int(Y.numel() * 4 * world),
@@ -454,6 +508,7 @@ def main():
             "e2e": e2e,
             "gpu_launches": launches * args.steps,
             "clocks": clocks.summary(),
+            **({"dry_run": f"{backend} backend, ranks share one GPU: not a measurement"} if backend != "nccl" else {}),
             "per_op_graph": secondary,
         }
         print(json.dumps(line), flush=True)

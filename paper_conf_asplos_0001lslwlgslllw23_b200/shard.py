@@ -16,6 +16,18 @@ from __future__ import annotations
 import torch
 
 
+def _all_gather(out: torch.Tensor, inp: torch.Tensor, group=None):
+    """all_gather_into_tensor; with a gloo group (CPU dry runs of the N > 1 path) the CUDA
+    tensors are staged through host memory."""
+    import torch.distributed as dist
+    if dist.get_backend(group) == "gloo" and out.is_cuda:
+        o = torch.empty(out.shape, dtype=out.dtype)
+        dist.all_gather_into_tensor(o, inp.cpu(), group=group)
+        out.copy_(o)
+    else:
+        dist.all_gather_into_tensor(out, inp, group=group)
+
+
 def block_rows(V: int, world: int) -> int:
     return -(-V // world)
 
@@ -59,7 +71,7 @@ class ShardedOperator:
         if self.world == 1:
             X_full.copy_(X_local)
         else:
-            dist.all_gather_into_tensor(X_full, X_local.contiguous(), group=self.group)
+            _all_gather(X_full, X_local.contiguous(), group=self.group)
         return X_full
 
     def edge_slice(self, T: torch.Tensor) -> torch.Tensor:
@@ -97,7 +109,7 @@ class ShardedOperator:
                 if self.world == 1:
                     bufs["full"][c].copy_(bufs["send"][c])
                 else:
-                    dist.all_gather_into_tensor(bufs["full"][c], bufs["send"][c], group=self.group)
+                    _all_gather(bufs["full"][c], bufs["send"][c], group=self.group)
                 bufs["ready"][c].record(side)
         for c, (c0, c1) in enumerate(bufs["cols"]):
             main.wait_event(bufs["ready"][c])
@@ -122,5 +134,5 @@ class ShardedOperator:
         pad = Y_local.new_zeros((m,) + tuple(Y_local.shape[1:]))
         pad[: Y_local.shape[0]].copy_(Y_local)
         allp = Y_local.new_empty((m * self.world,) + tuple(Y_local.shape[1:]))
-        dist.all_gather_into_tensor(allp, pad, group=self.group)
+        _all_gather(allp, pad, group=self.group)
         return torch.cat([allp[k * m: k * m + sizes[k]] for k in range(self.world)])
