@@ -72,7 +72,7 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
 }
 
 template <int KE, int GOP, int VEC, bool FAST>
-__global__ void __launch_bounds__(256) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
+__global__ void __launch_bounds__(256, (KE == K_COPY) ? 8 : 4) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
                                                int64_t n_chunks, int L_log2, int ftile, int n_tiles,
                                                float *__restrict__ scratch, int64_t sld) {
     constexpr int U = 4;                       // independent row gathers in flight per lane
