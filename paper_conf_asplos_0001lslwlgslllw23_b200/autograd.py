@@ -1,0 +1,101 @@
+"""Backward of the sum / mean aggregations through the same unified operator (SURVEY 8(f) f2:
+out-edge operators, "transposed aggregation for grad of copy_u_sum").
+
+The paper is inference-only; training needs get_outedges, i.e.
+the reversed graph.  Every backward step is again a graph operator of the 160-op set:
+  * d/dX of copy_u_sum(X)         = copy_u_sum over the reversed graph of dY
+  * d/dX of copy_u_mean(X)        = copy_u_sum over the reversed graph of dY / in_deg
+  * d/dX of u_mul_e_sum(X, w)     = u_mul_e_sum over the reversed graph of (dY, w)
+    (the reversed graph is built from the same COO with src / dst swapped, so edge ids -- and
+    hence the rows of w -- are unchanged)
+  * d/dw of u_mul_e_sum(X, w)     = u_dot_v message creation over the forward graph:
+    dw[e, h] = sum_{d in head h} X[src(e)][d] * dY[dst(e)][d]
+max / min backward (arg-max capture) is not provided.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+from . import Graph, op_run
+
+
+class GraphPair:
+    """A graph and its reverse (out-edge CSR), sharing edge ids."""
+
+    def __init__(self, num_vertices, src, dst):
+        self.V = int(num_vertices)
+        src = np.ascontiguousarray(src, dtype=np.int32)
+        dst = np.ascontiguousarray(dst, dtype=np.int32)
+        self.fwd = Graph(self.V, src, dst)
+        self.rev = Graph(self.V, dst, src)
+        self.in_deg = torch.from_numpy(np.bincount(dst, minlength=self.V).astype(np.float32))
+        self._inv_cache = {}
+
+    def inv_in_deg(self, device):
+        if device not in self._inv_cache:
+            d = self.in_deg.to(device)
+            self._inv_cache[device] = torch.where(d > 0, 1.0 / d.clamp(min=1), torch.zeros_like(d))[:, None]
+        return self._inv_cache[device]
+
+
+def _agg(graph, edge_op, gather_op, X, w=None, F=None, H=1):
+    F = F or X.shape[1]
+    Y = torch.empty(X.shape[0] if graph is None else graph.stats()["V"], F, device=X.device)
+    op_run(graph, edge_op, gather_op, A=X.contiguous(), a_type="u", B=None if w is None else w.contiguous(),
+           b_type=None if w is None else "e", C=Y, c_type="v", F=F, H=H)
+    return Y
+
+
+class _CopyUReduce(torch.autograd.Function):
+    @staticmethod
+    def forward(ctx, gp, X, mean):
+        ctx.gp, ctx.mean = gp, mean
+        return _agg(gp.fwd, "copy_lhs", "mean" if mean else "sum", X)
+
+    @staticmethod
+    def backward(ctx, dY):
+        gp = ctx.gp
+        g = dY.contiguous()
+        if ctx.mean:
+            g = g * gp.inv_in_deg(g.device)
+        return None, _agg(gp.rev, "copy_lhs", "sum", g), None
+
+
+class _UMulESum(torch.autograd.Function):
+    @staticmethod
+    def forward(ctx, gp, X, w):
+        ctx.gp = gp
+        ctx.save_for_backward(X, w)
+        H = w.shape[1]
+        return _agg(gp.fwd, "mul", "sum", X, w, H=H)
+
+    @staticmethod
+    def backward(ctx, dY):
+        gp = ctx.gp
+        X, w = ctx.saved_tensors
+        dY = dY.contiguous()
+        H = w.shape[1]
+        dX = dw = None
+        if ctx.needs_input_grad[1]:
+            dX = _agg(gp.rev, "mul", "sum", dY, w, H=H)
+        if ctx.needs_input_grad[2]:
+            dw = torch.empty(w.shape[0], H, device=w.device)
+            op_run(gp.fwd, "dot", "assign", A=X.contiguous(), a_type="u", B=dY, b_type="v", C=dw, c_type="e",
+                   F=X.shape[1], H=H)
+        return None, dX, dw
+
+
+def copy_u_sum(gp: GraphPair, X):
+    return _CopyUReduce.apply(gp, X, False)
+
+
+def copy_u_mean(gp: GraphPair, X):
+    return _CopyUReduce.apply(gp, X, True)
+
+
+def u_mul_e_sum(gp: GraphPair, X, w):
+    """w: [E, H] per-edge (per-head) weights; X: [V, F] with H | F."""
+    if w.dim() == 1:
+        w = w.view(-1, 1)
+    return _UMulESum.apply(gp, X, w)
