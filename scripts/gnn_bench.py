@@ -32,7 +32,7 @@ def torch_aggr(h, s, d, V, how):
 
 
 def build(model, fin, fout):
-    hid = HIDDEN[model]
+    hid = HIDDEN[model.split("_")[0]]
     if model == "GCN":
         return [gnn.GCNConv(fin, hid), gnn.GCNConv(hid, fout)]
     if model == "GIN":
