@@ -463,13 +463,19 @@ def main():
                       "pinned host X block -> device, all-gather, op, Y shard -> host, every step"}
 
     traffic = None
+    l2 = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
         try:
             ent = json.load(open(tp)).get(f"{args.config}:{args.op}:{F}:{chosen}")
             # dram__bytes_read.sum + dram__bytes_write.sum of one launch (ncu --set full)
             traffic = int(ent["dram_bytes_per_launch"]) if ent and world == 1 else None
-        except (ValueError, OSError):
+            if ent and world == 1 and "l2_to_sm_bytes" in ent:
+                # the binding roof of the tile-major schedule is L2 -> SM, not HBM
+                l2 = {"l2_to_sm_bytes_per_launch": int(ent["l2_to_sm_bytes"]),
+                      "achieved_gbs": round(ent["l2_to_sm_bytes"] / (kms * 1e-3) / 1e9, 1),
+                      "ncu_lts_throughput_pct": ent.get("lts_throughput_pct")}
+        except (ValueError, OSError, KeyError, TypeError):
             traffic = None
 
     secondary = None
@@ -503,7 +509,8 @@ def main():
                          "kernel": ("k_split per 64-column chunk, exchange overlapped" if chunked else
                                     "k_split (SV main traversal)" if chosen.startswith("SV") else "main traversal"),
                          "kernel_ms": round(kms, 4), "peak_source": peak_src,
-                         "bytes": "algorithmic (SURVEY 8(d)) per launch, this rank's rows"},
+                         "bytes": "algorithmic (SURVEY 8(d)) per launch, this rank's rows",
+                         "l2": l2},
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches * args.steps,
