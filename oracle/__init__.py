@@ -147,3 +147,31 @@ def partition(row_ptr, parts):
     out = np.zeros(parts + 1, dtype=np.int64)
     lib.ugo_partition(V, _ptr(row_ptr), int(parts), _ptr(out))
     return out
+
+
+def gat(V, src, dst, el, er, z, H, slope=0.2, bound=False):
+    """GAT attention chain by definition, fp64: edge softmax of
+    LeakyReLU(el_u + er_v) per head over each destination's in-edges, then the attention-weighted
+    sum of z_u.  el, er: [V, H]; z: [V, F] float32.  Returns (out [V, F], attn [E, H]) as float64,
+    plus the tolerance scale sum_e a |z| when bound=True."""
+    lib = _load()
+    if not hasattr(lib, "_gat_ready"):
+        p, i64, ci = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int
+        lib.ugo_gat.argtypes = [i64, i64, p, p, p, i64, p, i64, p, i64, ci, ci, ctypes.c_double, p, p, p]
+        lib.ugo_gat.restype = ci
+        lib._gat_ready = True
+    src = _c32(src)
+    dst = _c32(dst)
+    E = int(src.shape[0])
+    el = np.ascontiguousarray(el, dtype=np.float32).reshape(V, -1)
+    er = np.ascontiguousarray(er, dtype=np.float32).reshape(V, -1)
+    z = np.ascontiguousarray(z, dtype=np.float32)
+    F = int(z.shape[1])
+    out = np.zeros((V, F), dtype=np.float64)
+    attn = np.zeros((max(E, 1), H), dtype=np.float64)
+    bnd = np.zeros((V, F), dtype=np.float64) if bound else None
+    rc = lib.ugo_gat(V, E, _ptr(src), _ptr(dst), _ptr(el), el.shape[1], _ptr(er), er.shape[1],
+                     _ptr(z), F, F, int(H), float(slope), _ptr(out), _ptr(attn), _ptr(bnd))
+    if rc != 0:
+        raise ValueError(f"oracle rejected gat (F={F}, H={H}) rc={rc}")
+    return (out, attn[:E], bnd) if bound else (out, attn[:E])

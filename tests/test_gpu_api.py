@@ -83,7 +83,13 @@ def test_auto_selection_is_valid_for_every_class(c3):
         if go in ("max", "assign"):
             assert torch.equal(C, C2), (eo, go, s)
         else:
-            torch.testing.assert_close(C, C2, rtol=1e-5, atol=1e-5)
+            # both runs are within 1e-5 * sum|terms| of the exact sum (R11), so within 2e-5 of
+            # each other; atomic (edge-parallel) schedules sum in a run-dependent order
+            akw = {k: (v.abs() if torch.is_tensor(v) else v) for k, v in kw.items()}
+            S = torch.empty_like(C)
+            ug.op_run(g, eo, go, C=S, c_type=ct, F=32, H=1, schedule=s, **akw)
+            torch.cuda.synchronize()
+            assert ((C - C2).abs() <= 2e-5 * S).all(), (eo, go, s, (C - C2).abs().max().item())
 
 
 def test_prepared_op_and_cuda_graph_capture():
