@@ -277,9 +277,30 @@ def gat_chain_graph(ug, torch, dev, g, reps=50):
 
     eager = timed(lambda: [op() for op in chain])
     graph = timed(cg.replay)
+    # the same chain (with the real LeakyReLU / exp) as ONE traversal: ug_gat_attention (f3)
+    out, att = torch.empty(V, F, device=dev), torch.empty(E, H, device=dev)
+    fused = timed(lambda: ug.gat_attention(g, el, er, X, H, 0.2, out=out))
+    fused_attn = timed(lambda: ug.gat_attention(g, el, er, X, H, 0.2, out=out, attn=att))
+    dev_ts = []
+    for i in range(25):
+        torch.cuda._sleep(400_000)          # queued behind a spin kernel: device time only
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        ug.gat_attention(g, el, er, X, H, 0.2, out=out)
+        e1.record()
+        torch.cuda.synchronize()
+        if i >= 5:
+            dev_ts.append(e0.elapsed_time(e1) * 1e3)
+    # algorithmic bytes of the fused traversal: row_ptr, col_idx, el gathers (E x H), er (V x H),
+    # z gathers (E x F), out (V x F)
+    by = 4 * (V + 1) + 4 * E + 4 * E * H + 4 * V * H + 4 * E * F + 4 * V * F
+    dmed = statistics.median(dev_ts)
     return {"config": "C2", "op": "GAT attention chain (6 ops)", "F": F, "H": H,
             "schedules": [op.schedule for op in chain],
-            "eager_us_per_chain": round(eager, 2), "cuda_graph_us_per_chain": round(graph, 2)}
+            "eager_us_per_chain": round(eager, 2), "cuda_graph_us_per_chain": round(graph, 2),
+            "fused_one_kernel_us": round(fused, 2), "fused_with_attention_out_us": round(fused_attn, 2),
+            "fused_device_us": round(dmed, 2), "fused_logical_bytes": by,
+            "fused_gbs": round(by / (dmed * 1e-6) / 1e9, 1)}
 
 
 # ---------------------------------------------------------------------------- GPU run

@@ -207,6 +207,31 @@ ug_status ug_op_launch_count(const ug_graph *g, const ug_op_info *op, const ug_s
 ug_status ug_edge_permute(const ug_graph *g, const float *in, float *out, int32_t width,
                           void *stream);
 
+/*
+ * ug_gat_attention -- the GAT attention chain fused into ONE traversal.
+ * PAPER.md:224 lists GAT's graph operators: a message creation el_u + er_v (edge scores) and
+ * an aggregation-sum weighting each source feature by its edge weight; GAT's edge softmax
+ * between them (LeakyReLU, copy_e_max, e_sub_v + exp, copy_e_sum, e_div_v under the unified
+ * abstraction) is folded in.  For every destination v, head h < H and feature f = h*D + d
+ * (D = F / H), over v's in-edges e = (u -> v):
+ *     s(e,h)  = LeakyReLU(el[u][h] + er[v][h]) = s >= 0 ? s : slope * s
+ *     a(e,h)  = exp(s(e,h) - max_e' s(e',h)) / sum_e' exp(s(e',h) - max_e' s(e',h))
+ *     out[v][f] = sum_e a(e,h) * z[u][f]
+ *   el  [V_src][H] (ld_el), er [V][H] (ld_er), z [V_src][F] (ld_z): device fp32 inputs
+ *       (in a view: el, z by global src id; er by local row, as Src_V / Dst_V operands).
+ *   out [V][F] (ld_out): device fp32, every row written; zero in-degree rows -> 0 (R7).
+ *   attn: NULL, or device fp32 [E][H] (ld_attn) receiving a(e,h) at row = edge id (R9).
+ *   Accuracy: within 1e-5 * sum_e a(e,h) |z[u][f]| of the fp64 definition (oracle.gat);
+ *   attention within 1e-5 relative.  Deterministic (no atomics).  One kernel launch on
+ *   `stream`; the first call per graph uploads a small row list synchronously.
+ *   Errors: UG_ERR_INVALID_ARG (NULL graph / data, host-only graph), UG_ERR_SHAPE (H <= 0,
+ *   H does not divide F, ld < width), UG_ERR_OOM, UG_ERR_CUDA.
+ */
+ug_status ug_gat_attention(const ug_graph *g, const float *el, int64_t ld_el, const float *er,
+                           int64_t ld_er, const float *z, int64_t ld_z, int32_t F, int32_t H,
+                           float slope, float *out, int64_t ld_out, float *attn, int64_t ld_attn,
+                           void *stream);
+
 /* Schedule <-> text, Table 9 notation ("TE_G1_T16", "SV_G2048_F64"). */
 ug_status ug_schedule_parse(const char *text, ug_schedule *out);
 ug_status ug_schedule_format(const ug_schedule *s, char *buf, size_t len);

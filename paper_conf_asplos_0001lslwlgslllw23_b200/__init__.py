@@ -20,7 +20,7 @@ from ._ffi import (EDGE_OPS, GATHER_OPS, STRATEGIES, TTYPES, UgError, UgOpInfo, 
                    UgTensor, check, lib)
 
 __all__ = ["Graph", "op_run", "prepare", "PreparedOp", "schedule_select", "launch_count", "parse_schedule",
-           "format_schedule", "validate", "edge_permute", "selector_load", "UgError", "version"]
+           "format_schedule", "validate", "edge_permute", "selector_load", "gat_attention", "UgError", "version"]
 
 
 def version():
@@ -274,3 +274,34 @@ def edge_permute(graph, inp, out, stream=None):
 
 def selector_load(path):
     check(lib.ug_selector_load(str(path).encode()), "ug_selector_load")
+
+
+def _mat(x, name):
+    import torch
+    if not isinstance(x, torch.Tensor) or x.dtype != torch.float32 or not x.is_cuda:
+        raise TypeError(f"{name} must be a float32 CUDA tensor")
+    if x.dim() == 1:
+        x = x.view(-1, 1)
+    if x.dim() != 2 or (x.shape[1] > 1 and x.stride(1) != 1):
+        raise ValueError(f"{name} must be 2-D with unit column stride")
+    return x.data_ptr(), max(x.stride(0), x.shape[1])
+
+
+def gat_attention(graph, el, er, z, heads, slope=0.2, out=None, attn=None, stream=None):
+    """GAT attention chain in ONE traversal (ug_gat_attention):
+    out[v] = sum over in-edges e=(u->v) of softmax_e(LeakyReLU(el[u] + er[v])) per head * z[u].
+    el, er: [V, H]; z: [V, F] (H | F).  Returns out [V, F] (and fills attn [E, H] if given)."""
+    import torch
+    H = int(heads)
+    F = int(z.shape[1])
+    V = er.shape[0]
+    if out is None:
+        out = torch.empty(V, F, device=z.device, dtype=torch.float32)
+    pel, lel = _mat(el, "el")
+    per, ler = _mat(er, "er")
+    pz, lz = _mat(z, "z")
+    po, lo = _mat(out, "out")
+    pa, la = (None, 0) if attn is None else _mat(attn, "attn")
+    check(lib.ug_gat_attention(graph.handle, pel, lel, per, ler, pz, lz, F, H, float(slope), po, lo, pa, la,
+                               _current_stream(stream)), "ug_gat_attention")
+    return out

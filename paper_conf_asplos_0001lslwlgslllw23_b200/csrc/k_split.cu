@@ -1,235 +1,30 @@
-// k_split.cu -- Split-Vertex (SV), the B200 schedule for wide, skewed aggregations
-// (C3/C5).  It composes the paper's two knobs with two B200 facts: a
-// 126 MB L2 and 148 SMs that all want equal work.
-//
-//  * Row splitting (load balance): every destination row is cut into chunks of at most
-//    `group` in-edges (a hub of in-degree 4.9e4 becomes ~24 chunks).  A chunk is one work
-//    unit; rows with one chunk are owned and finalised in registers; the partial results
-//    of split rows go to a scratch slot and a fix-up kernel combines them in chunk order
-//    (deterministic; no atomics, no init pass).
-//  * Column tiles, tile-major (locality): the feature axis is cut into ftile-wide tiles and
-//    the grid is ordered tile-major, so at any time the gathered rows touch one
-//    V x ftile slab of X (C5, ftile 64: 60 MB) which stays L2-resident while the next
-//    slab streams in; each X element then comes from DRAM about once per tile pass
-//    instead of once per in-edge.
-//  * L = ftile / VEC lanes per unit (one VEC-wide feature chunk per lane), the in-edge loop
-//    unrolled 4x so each lane keeps 4 independent row gathers in flight.
-#include "k_dispatch.cuh"
+// k_split.cu -- SV launcher: dispatch on edge_op to the per-KE instantiations (k_split*.cu
+// split the instances over translation units so they compile in parallel).
+#include "k_split.cuh"
 
 namespace ug {
 
-// Inner in-edge loop of the SV fast path.  BM: 0 no B operand, 1 B is Dst_V (constant over
-// the row: loaded once), 2 / 3 B is an Edge tensor (row = CSR position) with per-head broadcast
-// / full width, 4 / 5 B is Src_V with broadcast / full width.  All offsets are 32-bit (the
-// host checks rows * ld < 2^32).  Advances k to the last multiple of UF.
-template <int KE, int GOP, int VEC, int BM>
-__device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t &k,
-                                                int64_t k1, int f, int64_t cb, float (&acc)[VEC]) {
-    // row gathers in flight per lane: 16 (measured +3 % over 8 on C5 at VEC 2), 8 for float4 rows
-    constexpr int UF = VEC == 4 ? 8 : 16;
-    const float *__restrict__ Ab = op.A.p;          // warp-uniform base
-    const uint64_t keep = l2_policy_evict_last();     // this tile's X column slab
-    const uint64_t stream = l2_policy_evict_first();  // col_idx / edge tensors: read once per pass
-    const uint32_t lda = (uint32_t)op.A.ld, fo = (uint32_t)f;
-    const uint32_t ldb = (uint32_t)op.B.ld, cbo = (uint32_t)cb;
-    constexpr bool bfull = BM == 3 || BM == 5;
-    float bconst[VEC];
-    if constexpr (BM == 1) fetch<VEC>(op.B, v, cb, bconst);
-    for (; k + UF <= k1; k += UF) {
-        uint32_t s[UF];
-#pragma unroll
-        for (int q = 0; q < UF; ++q) s[q] = (uint32_t)ldg_i32_hint(g.col + k + q, stream);
-        float m[UF][VEC];
-#pragma unroll
-        for (int q = 0; q < UF; ++q) ldg_vec_hint<VEC>(Ab + (s[q] * lda + fo), m[q], keep);
-        if constexpr (BM != 0) {
-#pragma unroll
-            for (int q = 0; q < UF; ++q) {
-                float b[VEC];
-                if constexpr (BM == 1) {
-#pragma unroll
-                    for (int i = 0; i < VEC; ++i) b[i] = bconst[i];
-                } else {
-                    const uint32_t row = (BM == 2 || BM == 3) ? (uint32_t)(k + q) : s[q];
-                    const float *bp = op.B.p + (row * ldb + cbo);
-                    if constexpr (bfull) {
-                        ldg_vec_hint<VEC>(bp, b, BM == 3 ? stream : keep);
-                    } else {
-                        const float x = __ldg(bp);
-#pragma unroll
-                        for (int i = 0; i < VEC; ++i) b[i] = x;
-                    }
-                }
-#pragma unroll
-                for (int i = 0; i < VEC; ++i) m[q][i] = edge_fn<KE>(m[q][i], b[i]);
-            }
-        }
-#pragma unroll
-        for (int q = 0; q < UF; ++q)
-#pragma unroll
-            for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[q][i]);
-    }
-}
-
-template <int KE, int GOP, int VEC, bool FAST>
-__global__ void __launch_bounds__(256, (KE == K_COPY) ? 8 : 4) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
-                                               int64_t n_chunks, int L_log2, int ftile, int n_tiles,
-                                               float *__restrict__ scratch, int64_t sld) {
-    constexpr int U = 4;                       // independent row gathers in flight per lane
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const int lane = (int)(t & ((1 << L_log2) - 1));
-    const int64_t u = t >> L_log2;
-    if (u >= n_chunks * n_tiles) return;
-    const int tile = (int)(u / n_chunks);
-    const int64_t c = u - (int64_t)tile * n_chunks;
-    const int f = tile * ftile + lane * VEC;
-    if (f >= op.W) return;
-    const int4 ch = chunks[c];
-    const int64_t v = ch.x;
-    const int64_t k1 = ch.z;
-    const int64_t ca = op_col(op.A, f);
-    const int64_t cb = op_col(op.B, f);
-
-    if constexpr (GOP == UG_GATHER_ASSIGN) {
-        for (int64_t k = ch.y; k < k1; ++k) {
-            const int64_t src = g.col[k];
-            const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
-            float m[VEC];
-            message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m);
-            st_out<VEC>(op.C + e * op.c_ld + f, m, op.W - f, op.c_vec);
-        }
-    } else {
-        float acc[VEC];
-#pragma unroll
-        for (int i = 0; i < VEC; ++i) acc[i] = g_init<GOP>();
-        int64_t k = ch.y;
-        if constexpr (FAST) {
-            // A is a full-width Src_V operand smaller than 4 GiB and edge ids are CSR positions:
-            // the row address is one IMAD + IMAD.WIDE from the (warp-uniform, L1-broadcast)
-            // column index, so each in-edge costs ~6 instructions per lane.  The B operand's
-            // addressing mode is resolved once per unit (a Dst_V operand is loaded once).
-            const int bfl = op.B.div == 1 ? 1 : 0;
-            const int bm = KE == K_COPY ? 0
-                         : op.B.type == UG_T_DST_V ? 1 : (op.B.type == UG_T_EDGE ? 2 + bfl : 4 + bfl);
-            if constexpr (KE == K_COPY) {
-                split_fast_loop<KE, GOP, VEC, 0>(g, op, v, k, k1, f, cb, acc);
-            } else {
-                switch (bm) {
-                case 1: split_fast_loop<KE, GOP, VEC, 1>(g, op, v, k, k1, f, cb, acc); break;
-                case 2: split_fast_loop<KE, GOP, VEC, 2>(g, op, v, k, k1, f, cb, acc); break;
-                case 3: split_fast_loop<KE, GOP, VEC, 3>(g, op, v, k, k1, f, cb, acc); break;
-                case 4: split_fast_loop<KE, GOP, VEC, 4>(g, op, v, k, k1, f, cb, acc); break;
-                default: split_fast_loop<KE, GOP, VEC, 5>(g, op, v, k, k1, f, cb, acc); break;
-                }
-            }
-        } else {
-            for (; k + U <= k1; k += U) {
-                float m[U][VEC];
-#pragma unroll
-                for (int q = 0; q < U; ++q) {
-                    const int64_t src = g.col[k + q];
-                    const int64_t e = g.eid ? (int64_t)g.eid[k + q] : k + q;
-                    message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m[q]);
-                }
-#pragma unroll
-                for (int q = 0; q < U; ++q)
-#pragma unroll
-                    for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[q][i]);
-            }
-        }
-        for (; k < k1; ++k) {
-            const int64_t src = g.col[k];
-            const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
-            float m[VEC];
-            message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m);
-#pragma unroll
-            for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[i]);
-        }
-        // outputs are written once: evict_first keeps them from displacing the X slab in L2
-        const uint64_t wpol = l2_policy_evict_first();
-        if (ch.w < 0) {
-            const int64_t deg = (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
-            float out[VEC];
-#pragma unroll
-            for (int i = 0; i < VEC; ++i) out[i] = g_finalize<GOP>(acc[i], deg);
-            if (f + VEC <= op.W && op.c_vec >= VEC) st_vec_hint<VEC>(op.C + v * op.c_ld + f, out, wpol);
-            else st_out<VEC>(op.C + v * op.c_ld + f, out, op.W - f, op.c_vec);
-        } else {
-            st_vec_hint<VEC>(scratch + (int64_t)ch.w * sld + f, acc, wpol);
-        }
-    }
-}
-
-// Fix-up of split rows: combine the row's partials in chunk order, finalise, store.
-template <int GOP, int VEC>
-__global__ void k_split_fix(GraphArgs g, OpArgs op, const int4 *__restrict__ split, int64_t n_split,
-                            const float *__restrict__ scratch, int64_t sld) {
-    const int64_t per_row = cdiv(op.W, VEC);
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (t >= n_split * per_row) return;
-    const int64_t r = t / per_row;
-    const int f = (int)(t - r * per_row) * VEC;
-    const int4 sp = split[r];
-    float acc[VEC];
-#pragma unroll
-    for (int i = 0; i < VEC; ++i) acc[i] = g_init<GOP>();
-    for (int s = 0; s < sp.z; ++s) {
-        float p[VEC];
-        ldg_vec<VEC>(scratch + (int64_t)(sp.y + s) * sld + f, p);
-#pragma unroll
-        for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], p[i]);
-    }
-    const int64_t v = sp.x;
-    const int64_t deg = (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
-#pragma unroll
-    for (int i = 0; i < VEC; ++i) acc[i] = g_finalize<GOP>(acc[i], deg);
-    st_out<VEC>(op.C + v * op.c_ld + f, acc, op.W - f, op.c_vec);
-}
+UG_SV_INSTANTIATE(K_COPY)
+// instantiated in k_split_addsub.cu / k_split_mul.cu / k_split_div.cu
+extern template cudaError_t launch_split_ke<K_ADD>(int, const GraphArgs &, const OpArgs &, const LaunchCfg &,
+                                                   const SplitPlan &, float *, cudaStream_t, cudaEvent_t, cudaEvent_t);
+extern template cudaError_t launch_split_ke<K_SUB>(int, const GraphArgs &, const OpArgs &, const LaunchCfg &,
+                                                   const SplitPlan &, float *, cudaStream_t, cudaEvent_t, cudaEvent_t);
+extern template cudaError_t launch_split_ke<K_MUL>(int, const GraphArgs &, const OpArgs &, const LaunchCfg &,
+                                                   const SplitPlan &, float *, cudaStream_t, cudaEvent_t, cudaEvent_t);
+extern template cudaError_t launch_split_ke<K_DIV>(int, const GraphArgs &, const OpArgs &, const LaunchCfg &,
+                                                   const SplitPlan &, float *, cudaStream_t, cudaEvent_t, cudaEvent_t);
 
 cudaError_t launch_split_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
                                 const LaunchCfg &c, const SplitPlan &plan, float *scratch,
                                 cudaStream_t s, cudaEvent_t ev_begin, cudaEvent_t ev_end) {
-    const int L = c.ftile / c.vec;
-    const int n_tiles = (int)cdiv(op.W, c.ftile);
-    const int64_t threads = plan.n_chunks * n_tiles * (int64_t)L;
-    if (threads == 0) return cudaSuccess;
-    const int64_t grid = cdiv(threads, c.block);
-    const int L_log2 = ilog2(L);
-    const int64_t sld = cdiv(op.W, 4) * 4;
-    const int4 *chunks = reinterpret_cast<const int4 *>(plan.d_chunk);
-    if (ev_begin) cudaEventRecord(ev_begin, s);
-    // fast path: full-width Src_V operand whose rows are byte-addressable in 32 bits
-    // (V_total * ld * 4 < 2^32; the host passes the bound in op.A.ld via g.V_src), identity eids
-    // fast path: full-width Src_V A operand, identity edge ids, and every operand row
-    // addressable with 32-bit element offsets (rows * ld < 2^32)
-    const uint64_t lim = 1ull << 32;
-    bool fast = op.A.type == UG_T_SRC_V && op.A.div == 1 && g.eid == nullptr &&
-                (uint64_t)g.V_src * (uint64_t)op.A.ld < lim;
-    if (kedge != K_COPY) {
-        const uint64_t brows = op.B.type == UG_T_EDGE ? (uint64_t)g.E : (uint64_t)g.V_src;
-        fast = fast && brows * (uint64_t)op.B.ld < lim;
+    switch (kedge) {
+    case K_COPY: return launch_split_ke<K_COPY>(gather, g, op, c, plan, scratch, s, ev_begin, ev_end);
+    case K_ADD: return launch_split_ke<K_ADD>(gather, g, op, c, plan, scratch, s, ev_begin, ev_end);
+    case K_SUB: return launch_split_ke<K_SUB>(gather, g, op, c, plan, scratch, s, ev_begin, ev_end);
+    case K_MUL: return launch_split_ke<K_MUL>(gather, g, op, c, plan, scratch, s, ev_begin, ev_end);
+    default: return launch_split_ke<K_DIV>(gather, g, op, c, plan, scratch, s, ev_begin, ev_end);
     }
-    UG_DISPATCH_VEC(c.vec, VEC,
-        UG_DISPATCH_KE(kedge, KE,
-            UG_DISPATCH_GOP(gather, GOP, {
-                if (fast)
-                    k_split<KE, GOP, VEC, true><<<(unsigned)grid, c.block, 0, s>>>(
-                        g, op, chunks, plan.n_chunks, L_log2, c.ftile, n_tiles, scratch, sld);
-                else
-                    k_split<KE, GOP, VEC, false><<<(unsigned)grid, c.block, 0, s>>>(
-                        g, op, chunks, plan.n_chunks, L_log2, c.ftile, n_tiles, scratch, sld);
-            })));
-    if (ev_end) cudaEventRecord(ev_end, s);
-    cudaError_t err = cudaGetLastError();
-    if (err != cudaSuccess || gather == UG_GATHER_ASSIGN || plan.n_split_rows == 0) return err;
-    const int64_t per_row = cdiv(op.W, c.vec);
-    const int64_t fgrid = cdiv(plan.n_split_rows * per_row, 256);
-    const int4 *split = reinterpret_cast<const int4 *>(plan.d_split);
-    UG_DISPATCH_VEC(c.vec, VEC,
-        UG_DISPATCH_RED(gather, GOP,
-            k_split_fix<GOP, VEC><<<(unsigned)fgrid, 256, 0, s>>>(g, op, split, plan.n_split_rows,
-                                                                  scratch, sld)));
-    return cudaGetLastError();
 }
 
 }  // namespace ug

@@ -1,0 +1,266 @@
+// k_split.cuh -- Split-Vertex (SV), the B200 schedule for wide, skewed aggregations
+// (C3/C5).  It composes the paper's two knobs with two B200 facts: a
+// 126 MB L2 and 148 SMs that all want equal work.
+//
+//  * Row splitting (load balance): every destination row is cut into chunks of at most
+//    `group` in-edges (a hub of in-degree 4.9e4 becomes ~24 chunks).  A chunk is one work
+//    unit; rows with one chunk are owned and finalised in registers; the partial results
+//    of split rows go to a scratch slot and a fix-up kernel combines them in chunk order
+//    (deterministic; no atomics, no init pass).
+//  * Column tiles, tile-major (locality): the feature axis is cut into ftile-wide tiles and
+//    the grid is ordered tile-major, so at any time the gathered rows touch one
+//    V x ftile slab of X (C5, ftile 64: 60 MB) which stays L2-resident while the next
+//    slab streams in; each X element then comes from DRAM about once per tile pass
+//    instead of once per in-edge.
+//  * L = ftile / VEC lanes per unit (one VEC-wide feature chunk per lane), the in-edge loop
+//    unrolled 4x so each lane keeps 4 independent row gathers in flight.
+#pragma once
+#include <type_traits>
+#include "k_dispatch.cuh"
+
+namespace ug {
+
+// Inner in-edge loop of the SV fast path.  BM: 0 no B operand, 1 B is Dst_V (constant over
+// the row: loaded once), 2 / 3 B is an Edge tensor (row = CSR position) with per-head broadcast
+// / full width, 4 / 5 B is Src_V with broadcast / full width.  All offsets are 32-bit (the
+// host checks rows * ld < 2^32).  The last, partial group of UF edges is predicated (its
+// missing slots re-read the row's last edge, an L1 hit, and are not combined), so short rows
+// never fall into a serial one-edge-at-a-time tail.  Advances k to k1.
+template <int KE, int GOP, int VEC, int BM>
+__device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t &k,
+                                                int64_t k1, int f, int64_t cb, float (&acc)[VEC]) {
+    // row gathers in flight per lane: 16 (measured +3 % over 8 on C5 at VEC 2), 8 for float4 rows;
+    // half that when a B operand is loaded per edge (register budget of 40 for 6 CTAs / SM)
+#ifndef UG_BM2_UF
+#define UG_BM2_UF (VEC == 4 ? 4 : 8)
+#endif
+    constexpr int UF = BM == 0 || BM == 1 ? (VEC == 4 ? 8 : 16)
+                     : (BM == 2 && KE != K_DIV) ? UG_BM2_UF : (VEC == 4 ? 4 : 8) / (KE == K_DIV ? 2 : 1);
+    const float *__restrict__ Ab = op.A.p;          // warp-uniform base
+    const uint64_t keep = l2_policy_evict_last();     // this tile's X column slab
+    const uint64_t stream = l2_policy_evict_first();  // col_idx / edge tensors: read once per pass
+    const uint32_t lda = (uint32_t)op.A.ld, fo = (uint32_t)f;
+    const uint32_t ldb = (uint32_t)op.B.ld, cbo = (uint32_t)cb;
+    constexpr bool bfull = BM == 3 || BM == 5;
+    float bconst[VEC];
+    if constexpr (BM == 1) fetch<VEC>(op.B, v, cb, bconst);
+    const int64_t kl = k1 - 1;
+    auto group = [&](auto pred_tag, auto n_tag) {
+        constexpr bool PRED = decltype(pred_tag)::value;
+        constexpr int UF = decltype(n_tag)::value;
+        uint32_t s[UF];
+#pragma unroll
+        for (int q = 0; q < UF; ++q) s[q] = (uint32_t)ldg_i32_hint(g.col + (PRED ? min(k + q, kl) : k + q), stream);
+        float m[UF][VEC];
+#pragma unroll
+        for (int q = 0; q < UF; ++q) ldg_vec_hint<VEC>(Ab + (s[q] * lda + fo), m[q], keep);
+        if constexpr (BM != 0) {
+#pragma unroll
+            for (int q = 0; q < UF; ++q) {
+                float b[VEC];
+                if constexpr (BM == 1) {
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) b[i] = bconst[i];
+                } else {
+                    const uint32_t row = (BM == 2 || BM == 3) ? (uint32_t)(PRED ? min(k + q, kl) : k + q) : s[q];
+                    const float *bp = op.B.p + (row * ldb + cbo);
+                    if constexpr (bfull) {
+                        ldg_vec_hint<VEC>(bp, b, BM == 3 ? stream : keep);
+                    } else {
+                        const float x = __ldg(bp);
+#pragma unroll
+                        for (int i = 0; i < VEC; ++i) b[i] = x;
+                    }
+                }
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) m[q][i] = edge_fn<KE>(m[q][i], b[i]);
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < UF; ++q) {
+            const bool ok = !PRED || k + q < k1;
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) acc[i] = ok ? g_combine<GOP>(acc[i], m[q][i]) : acc[i];
+        }
+    };
+    for (; k + UF <= k1; k += UF) group(std::false_type{}, std::integral_constant<int, UF>{});
+    // the last, partial group: predicated half-groups (fewer registers), not a serial tail
+    constexpr int UH = UF / 2 > 0 ? UF / 2 : 1;
+    for (; k < k1; k += UH) group(std::true_type{}, std::integral_constant<int, UH>{});
+    k = k1;
+}
+
+// BM < 0: generic addressing (any operand types, eid); BM >= 0: the fast path with the B
+// operand's addressing mode fixed at compile time (see split_fast_loop).
+template <int KE, int GOP, int VEC, int BM>
+#ifndef UG_BM2_MINB
+#define UG_BM2_MINB 5
+#endif
+__global__ void __launch_bounds__(256, (BM == 0) ? 8 : (BM == 2 ? UG_BM2_MINB : (BM > 0 ? (VEC == 4 ? 5 : 6) : 4))) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
+                                               int64_t n_chunks, int L_log2, int ftile, int n_tiles,
+                                               float *__restrict__ scratch, int64_t sld) {
+    constexpr bool FAST = BM >= 0;
+    constexpr int U = 4;                       // independent row gathers in flight per lane
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int lane = (int)(t & ((1 << L_log2) - 1));
+    const int64_t u = t >> L_log2;
+    if (u >= n_chunks * n_tiles) return;
+    const int tile = (int)(u / n_chunks);
+    const int64_t c = u - (int64_t)tile * n_chunks;
+    const int f = tile * ftile + lane * VEC;
+    if (f >= op.W) return;
+    const int4 ch = chunks[c];
+    const int64_t v = ch.x;
+    const int64_t k1 = ch.z;
+    const int64_t ca = op_col(op.A, f);
+    const int64_t cb = op_col(op.B, f);
+
+    if constexpr (GOP == UG_GATHER_ASSIGN) {
+        for (int64_t k = ch.y; k < k1; ++k) {
+            const int64_t src = g.col[k];
+            const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
+            float m[VEC];
+            message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m);
+            st_out<VEC>(op.C + e * op.c_ld + f, m, op.W - f, op.c_vec);
+        }
+    } else {
+        float acc[VEC];
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) acc[i] = g_init<GOP>();
+        int64_t k = ch.y;
+        if constexpr (FAST) {
+            // A is a full-width Src_V operand smaller than 4 GiB and edge ids are CSR positions:
+            // the row address is one IMAD + IMAD.WIDE from the (warp-uniform, L1-broadcast)
+            // column index, so each in-edge costs ~6 instructions per lane.  The B operand's
+            // addressing mode BM is a template parameter (a Dst_V operand is loaded once).
+            split_fast_loop<KE, GOP, VEC, BM>(g, op, v, k, k1, f, cb, acc);
+        } else {
+            for (; k + U <= k1; k += U) {
+                float m[U][VEC];
+#pragma unroll
+                for (int q = 0; q < U; ++q) {
+                    const int64_t src = g.col[k + q];
+                    const int64_t e = g.eid ? (int64_t)g.eid[k + q] : k + q;
+                    message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m[q]);
+                }
+#pragma unroll
+                for (int q = 0; q < U; ++q)
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[q][i]);
+            }
+        }
+        for (; k < k1; ++k) {
+            const int64_t src = g.col[k];
+            const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
+            float m[VEC];
+            message<KE, VEC>(op, op_row(op.A.type, src, v, e), ca, op_row(op.B.type, src, v, e), cb, m);
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], m[i]);
+        }
+        // outputs are written once: evict_first keeps them from displacing the X slab in L2
+        const uint64_t wpol = l2_policy_evict_first();
+        if (ch.w < 0) {
+            const int64_t deg = (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
+            float out[VEC];
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) out[i] = g_finalize<GOP>(acc[i], deg);
+            if (f + VEC <= op.W && op.c_vec >= VEC) st_vec_hint<VEC>(op.C + v * op.c_ld + f, out, wpol);
+            else st_out<VEC>(op.C + v * op.c_ld + f, out, op.W - f, op.c_vec);
+        } else {
+            st_vec_hint<VEC>(scratch + (int64_t)ch.w * sld + f, acc, wpol);
+        }
+    }
+}
+
+// Fix-up of split rows: combine the row's partials in chunk order, finalise, store.
+template <int GOP, int VEC>
+__global__ void k_split_fix(GraphArgs g, OpArgs op, const int4 *__restrict__ split, int64_t n_split,
+                            const float *__restrict__ scratch, int64_t sld) {
+    const int64_t per_row = cdiv(op.W, VEC);
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= n_split * per_row) return;
+    const int64_t r = t / per_row;
+    const int f = (int)(t - r * per_row) * VEC;
+    const int4 sp = split[r];
+    float acc[VEC];
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) acc[i] = g_init<GOP>();
+    for (int s = 0; s < sp.z; ++s) {
+        float p[VEC];
+        ldg_vec<VEC>(scratch + (int64_t)(sp.y + s) * sld + f, p);
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], p[i]);
+    }
+    const int64_t v = sp.x;
+    const int64_t deg = (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) acc[i] = g_finalize<GOP>(acc[i], deg);
+    st_out<VEC>(op.C + v * op.c_ld + f, acc, op.W - f, op.c_vec);
+}
+
+// Launch of one edge_op's SV instances (explicitly instantiated per KE in k_split*.cu).
+template <int KE>
+cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, const LaunchCfg &c,
+                            const SplitPlan &plan, float *scratch, cudaStream_t s, cudaEvent_t ev_begin,
+                            cudaEvent_t ev_end) {
+    const int L = c.ftile / c.vec;
+    const int n_tiles = (int)cdiv(op.W, c.ftile);
+    const int64_t threads = plan.n_chunks * n_tiles * (int64_t)L;
+    if (threads == 0) return cudaSuccess;
+    const int64_t grid = cdiv(threads, c.block);
+    const int L_log2 = ilog2(L);
+    const int64_t sld = cdiv(op.W, 4) * 4;
+    const int4 *chunks = reinterpret_cast<const int4 *>(plan.d_chunk);
+    if (ev_begin) cudaEventRecord(ev_begin, s);
+    // fast path: full-width Src_V A operand, identity edge ids, and every operand row
+    // addressable with 32-bit element offsets (rows * ld < 2^32)
+    const uint64_t lim = 1ull << 32;
+    bool fast = op.A.type == UG_T_SRC_V && op.A.div == 1 && g.eid == nullptr &&
+                (uint64_t)g.V_src * (uint64_t)op.A.ld < lim && gather != UG_GATHER_ASSIGN;
+    if (KE != K_COPY) {
+        const uint64_t brows = op.B.type == UG_T_EDGE ? (uint64_t)g.E : (uint64_t)g.V_src;
+        fast = fast && brows * (uint64_t)op.B.ld < lim;
+    }
+    const int bfl = op.B.div == 1 ? 1 : 0;
+    const int bm = !fast ? -1 : KE == K_COPY ? 0
+                 : op.B.type == UG_T_DST_V ? 1 : (op.B.type == UG_T_EDGE ? 2 + bfl : 4 + bfl);
+#define UG_SV_LAUNCH(BMV)                                                                               \
+    k_split<KE, GOP, VEC, BMV><<<(unsigned)grid, c.block, 0, s>>>(g, op, chunks, plan.n_chunks, L_log2, \
+                                                                 c.ftile, n_tiles, scratch, sld)
+    UG_DISPATCH_VEC(c.vec, VEC,
+        UG_DISPATCH_GOP(gather, GOP, {
+            if constexpr (GOP == UG_GATHER_ASSIGN) {
+                UG_SV_LAUNCH(-1);
+            } else if constexpr (KE == K_COPY) {
+                if (bm == 0) UG_SV_LAUNCH(0); else UG_SV_LAUNCH(-1);
+            } else {
+                switch (bm) {
+                case 1: UG_SV_LAUNCH(1); break;
+                case 2: UG_SV_LAUNCH(2); break;
+                case 3: UG_SV_LAUNCH(3); break;
+                case 4: UG_SV_LAUNCH(4); break;
+                case 5: UG_SV_LAUNCH(5); break;
+                default: UG_SV_LAUNCH(-1); break;
+                }
+            }
+        }));
+#undef UG_SV_LAUNCH
+    if (ev_end) cudaEventRecord(ev_end, s);
+    cudaError_t err = cudaGetLastError();
+    if (err != cudaSuccess || gather == UG_GATHER_ASSIGN || plan.n_split_rows == 0) return err;
+    const int64_t per_row = cdiv(op.W, c.vec);
+    const int64_t fgrid = cdiv(plan.n_split_rows * per_row, 256);
+    const int4 *split = reinterpret_cast<const int4 *>(plan.d_split);
+    UG_DISPATCH_VEC(c.vec, VEC,
+        UG_DISPATCH_RED(gather, GOP,
+            k_split_fix<GOP, VEC><<<(unsigned)fgrid, 256, 0, s>>>(g, op, split, plan.n_split_rows,
+                                                                  scratch, sld)));
+    return cudaGetLastError();
+}
+
+#define UG_SV_INSTANTIATE(KE)                                                                            \
+    template cudaError_t launch_split_ke<KE>(int, const GraphArgs &, const OpArgs &, const LaunchCfg &, \
+                                             const SplitPlan &, float *, cudaStream_t, cudaEvent_t,     \
+                                             cudaEvent_t);
+
+}  // namespace ug

@@ -64,6 +64,7 @@ struct SplitPlan {
     int64_t n_split_chunks = 0; // chunks belonging to split rows (scratch slots)
     int32_t *d_chunk = nullptr;   // [n_chunks] x 4 int32: row, k0, k1, scratch slot (-1 = owner)
     int32_t *d_split = nullptr;   // [n_split_rows] x 4 int32: row, first slot, n slots, 0
+    int32_t *d_slot_row = nullptr; // [n_split_chunks]: index into d_split of the slot's row
 };
 
 // Kernel launchers (kernels/*.cu).  All return cudaGetLastError().
@@ -80,6 +81,18 @@ cudaError_t launch_dot(bool vertex_units, int gather, const GraphArgs &g, const 
                        const LaunchCfg &c, cudaStream_t s);
 cudaError_t launch_init(int gather, const OpArgs &op, int64_t rows, cudaStream_t s);
 cudaError_t launch_epilogue(int gather, const GraphArgs &g, const OpArgs &op, cudaStream_t s);
+// Fused GAT attention chain (ug_gat_attention, k_gat.cu).
+struct GatArgs {
+    const float *el, *er, *z;   // [V_src][H], [V][H] (local rows), [V_src][F]
+    int64_t ld_el, ld_er, ld_z;
+    float *out, *attn;          // [V][F] (local rows); attn [E][H] by edge id or NULL
+    int64_t ld_out, ld_attn;
+    int32_t F, H, D;
+    float slope;
+};
+cudaError_t launch_gat(const GraphArgs &g, const GatArgs &a, int vec, int L, const SplitPlan &plan,
+                       const int32_t *slot_row, float *sacc, float *sst, int64_t sld, int64_t nfc,
+                       int32_t *counters, cudaStream_t s);
 cudaError_t launch_permute(const int32_t *eid, const float *in, float *out, int64_t E, int width,
                            cudaStream_t s);
 
@@ -118,5 +131,8 @@ struct ug_graph {
     // UG_SV plans keyed by chunk size.
     mutable std::mutex mu;
     mutable std::map<int, ug::SplitPlan> plans;
+    // per-(split row, column tile) arrival counters of single-launch split-row merges
+    // (ug_gat_attention), keyed by chunk size * 65536 + column tiles; zero between calls
+    mutable std::map<int64_t, int32_t *> counters;
     mutable std::vector<void *> plan_allocs;
 };

@@ -194,7 +194,7 @@ static ug_status get_plan(const ug_graph *g, int G, const SplitPlan **out) {
     std::lock_guard<std::mutex> lock(g->mu);
     auto it = g->plans.find(G);
     if (it != g->plans.end()) { *out = &it->second; return UG_OK; }
-    std::vector<int32_t> chunks, split;
+    std::vector<int32_t> chunks, split, slot_row;
     int64_t slot = 0;
     for (int64_t v = 0; v < g->V; ++v) {
         const int64_t k0 = (int64_t)g->h_row_ptr[v] - g->e0, k1 = (int64_t)g->h_row_ptr[v + 1] - g->e0;
@@ -205,6 +205,7 @@ static ug_status get_plan(const ug_graph *g, int G, const SplitPlan **out) {
             split.insert(split.end(), {(int32_t)v, (int32_t)slot, (int32_t)n, 0});
             for (int64_t i = 0; i < n; ++i) {
                 const int64_t a = k0 + i * G, b = std::min(k1, a + G);
+                slot_row.push_back((int32_t)(split.size() / 4 - 1));
                 chunks.insert(chunks.end(), {(int32_t)v, (int32_t)a, (int32_t)b, (int32_t)slot++});
             }
         }
@@ -213,17 +214,21 @@ static ug_status get_plan(const ug_graph *g, int G, const SplitPlan **out) {
     p.n_chunks = (int64_t)chunks.size() / 4;
     p.n_split_rows = (int64_t)split.size() / 4;
     p.n_split_chunks = slot;
-    void *dc = nullptr, *ds = nullptr;
+    void *dc = nullptr, *ds = nullptr, *dr = nullptr;
     if (cudaMalloc(&dc, std::max<size_t>(16, chunks.size() * 4)) != cudaSuccess ||
-        cudaMalloc(&ds, std::max<size_t>(16, split.size() * 4)) != cudaSuccess)
+        cudaMalloc(&ds, std::max<size_t>(16, split.size() * 4)) != cudaSuccess ||
+        cudaMalloc(&dr, std::max<size_t>(16, slot_row.size() * 4)) != cudaSuccess)
         return set_error(UG_ERR_OOM, "SV plan allocation failed");
     g->plan_allocs.push_back(dc);
     g->plan_allocs.push_back(ds);
+    g->plan_allocs.push_back(dr);
     if ((!chunks.empty() && cudaMemcpy(dc, chunks.data(), chunks.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) ||
-        (!split.empty() && cudaMemcpy(ds, split.data(), split.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess))
+        (!split.empty() && cudaMemcpy(ds, split.data(), split.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess) ||
+        (!slot_row.empty() && cudaMemcpy(dr, slot_row.data(), slot_row.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess))
         return set_error(UG_ERR_CUDA, "SV plan upload failed");
     p.d_chunk = (int32_t *)dc;
     p.d_split = (int32_t *)ds;
+    p.d_slot_row = (int32_t *)dr;
     auto res = g->plans.emplace(G, p);
     *out = &res.first->second;
     return UG_OK;
@@ -442,3 +447,79 @@ extern "C" const char *ug_status_string(ug_status s) {
 extern "C" const char *ug_last_error(void) { return g_last_error.c_str(); }
 
 extern "C" const char *ug_version(void) { return "ugraph-b200 0.1 (sm_100a)"; }
+
+// ------------------------------------------------------------------------- fused GAT chain
+namespace ug {
+// Arrival counters for single-launch split-row merges: n_split_rows x n_tiles int32, zeroed
+// once (synchronously) at first use; every call leaves them zero again.
+static ug_status get_counters(const ug_graph *g, int G, int n_tiles, int64_t n_split_rows, int32_t **out) {
+    std::lock_guard<std::mutex> lock(g->mu);
+    const int64_t key = (int64_t)G * 65536 + n_tiles;
+    auto it = g->counters.find(key);
+    if (it != g->counters.end()) { *out = it->second; return UG_OK; }
+    void *d = nullptr;
+    const size_t bytes = std::max<size_t>(16, (size_t)n_split_rows * n_tiles * 4);
+    if (cudaMalloc(&d, bytes) != cudaSuccess) return set_error(UG_ERR_OOM, "counter allocation failed");
+    g->plan_allocs.push_back(d);
+    if (cudaMemset(d, 0, bytes) != cudaSuccess) return set_error(UG_ERR_CUDA, "counter init failed");
+    g->counters.emplace(key, (int32_t *)d);
+    *out = (int32_t *)d;
+    return UG_OK;
+}
+
+static bool aligned(const void *p, int64_t ld, int vec) {
+    return ((uintptr_t)p % (4 * vec)) == 0 && ld % vec == 0;
+}
+}  // namespace ug
+
+extern "C" ug_status ug_gat_attention(const ug_graph *g, const float *el, int64_t ld_el, const float *er,
+                                      int64_t ld_er, const float *z, int64_t ld_z, int32_t F, int32_t H,
+                                      float slope, float *out, int64_t ld_out, float *attn, int64_t ld_attn,
+                                      void *stream) {
+    using namespace ug;
+    if (!g) return set_error(UG_ERR_INVALID_ARG, "ug_gat_attention: NULL graph");
+    if (g->host_only) return set_error(UG_ERR_INVALID_ARG, "ug_gat_attention needs a device graph");
+    if (F <= 0 || H <= 0 || F % H != 0) return set_error(UG_ERR_SHAPE, "ug_gat_attention: need F > 0, H > 0, H | F");
+    if (ld_el < H || ld_er < H || ld_z < F || ld_out < F || (attn && ld_attn < H))
+        return set_error(UG_ERR_SHAPE, "ug_gat_attention: ld < width");
+    if (g->V > 0 && (!er || !out)) return set_error(UG_ERR_INVALID_ARG, "ug_gat_attention: NULL er / out");
+    if (g->E > 0 && (!el || !z)) return set_error(UG_ERR_INVALID_ARG, "ug_gat_attention: NULL el / z");
+    if (g->V == 0) return UG_OK;
+    const int D = F / H;
+    int vec = 4;
+    while (vec > 1 && (D % vec != 0 || !aligned(z, ld_z, vec) || !aligned(out, ld_out, vec))) vec >>= 1;
+    int L = 1;
+    while (L < 32 && (int64_t)L * vec < F) L <<= 1;
+    const int n_tiles = (F + L * vec - 1) / (L * vec);
+    // rows are cut into chunks of <= G in-edges (the SV plan): latency of the longest chunk
+    // vs. merge overhead; UG_GAT_CHUNK overrides (experiments)
+    int G = 32;
+    if (const char *ev = std::getenv("UG_GAT_CHUNK")) G = std::max(1, std::atoi(ev));
+    const SplitPlan *plan = nullptr;
+    ug_status st = get_plan(g, G, &plan);
+    if (st != UG_OK) return st;
+    if (plan->n_chunks * n_tiles >= (int64_t)1 << 31)
+        return set_error(UG_ERR_SHAPE, "ug_gat_attention: more than 2^31 (chunk, tile) units");
+    int32_t *counters = nullptr;
+    if ((st = get_counters(g, G, n_tiles, plan->n_split_rows, &counters)) != UG_OK) return st;
+    GatArgs a;
+    a.el = el; a.er = er; a.z = z;
+    a.ld_el = ld_el; a.ld_er = ld_er; a.ld_z = ld_z;
+    a.out = out; a.attn = attn; a.ld_out = ld_out; a.ld_attn = ld_attn;
+    a.F = F; a.H = H; a.D = D; a.slope = slope;
+    cudaStream_t s = (cudaStream_t)stream;
+    const int64_t sld = (F + 3) / 4 * 4, nfc = (F + vec - 1) / vec;
+    float *scratch = nullptr;
+    if (plan->n_split_chunks > 0) {
+        ensure_pool_retains();
+        const size_t bytes = sizeof(float) * (size_t)plan->n_split_chunks * (size_t)(sld + 2 * nfc);
+        if (cudaMallocAsync((void **)&scratch, bytes, s) != cudaSuccess)
+            return set_error(UG_ERR_OOM, "ug_gat_attention: scratch allocation failed");
+    }
+    float *sst = scratch ? scratch + plan->n_split_chunks * sld : nullptr;
+    cudaError_t e = launch_gat(graph_args(g), a, vec, L, *plan, plan->d_slot_row, scratch, sst, sld, nfc,
+                               counters, s);
+    if (scratch) cudaFreeAsync(scratch, s);
+    if (e != cudaSuccess) return set_error(UG_ERR_CUDA, std::string("ug_gat_attention: ") + cudaGetErrorString(e));
+    return UG_OK;
+}
