@@ -175,3 +175,35 @@ def gat(V, src, dst, el, er, z, H, slope=0.2, bound=False):
     if rc != 0:
         raise ValueError(f"oracle rejected gat (F={F}, H={H}) rc={rc}")
     return (out, attn[:E], bnd) if bound else (out, attn[:E])
+
+
+def op_arg(V, src, dst, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, F=None, H=1):
+    """Max/min aggregation with arg capture: returns (C [V, F] float32,
+    arg [V, F] int64 edge ids, -1 for zero in-degree rows); ties keep the first edge id."""
+    lib = _load()
+    if not hasattr(lib, "_arg_ready"):
+        p, i64, ci = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int
+        lib.ugo_op_arg.argtypes = [i64, i64, p, p, ci, ci, p, ci, ci, i64, p, ci, ci, i64, p, i64, ci, ci, p, i64]
+        lib.ugo_op_arg.restype = ci
+        lib._arg_ready = True
+    src = _c32(src)
+    dst = _c32(dst)
+    E = int(src.shape[0])
+    ops = []
+    for X in (A, B):
+        if X is None:
+            ops.append((None, 1, 0))
+        else:
+            X = np.ascontiguousarray(X, dtype=np.float32)
+            if X.ndim == 1:
+                X = X.reshape(-1, 1)
+            ops.append((X, X.shape[1], X.shape[1]))
+    (Aa, aw, ald), (Ba, bw, bld) = ops
+    C = np.zeros((V, F), dtype=np.float32)
+    arg = np.zeros((V, F), dtype=np.int64)
+    rc = lib.ugo_op_arg(V, E, _ptr(src), _ptr(dst), EDGE_OPS[edge_op], GATHER_OPS[gather_op],
+                        _ptr(Aa), TYPES[a_type], aw, ald, _ptr(Ba), TYPES[b_type], bw, bld,
+                        _ptr(C), F, int(F), int(H), _ptr(arg), F)
+    if rc != 0:
+        raise ValueError(f"oracle rejected arg op ({edge_op},{gather_op}) rc={rc}")
+    return C, arg
