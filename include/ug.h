@@ -232,6 +232,33 @@ ug_status ug_gat_attention(const ug_graph *g, const float *el, int64_t ld_el, co
                            float slope, float *out, int64_t ld_out, float *attn, int64_t ld_attn,
                            void *stream);
 
+/*
+ * ug_op_run_arg -- a max/min aggregation with arg capture (training of
+ * GraphSAGE-max style layers: the paper itself is inference-only).
+ * Computes C exactly as ug_op_run would (bit-identical values) for op_info with gather
+ * max/min, C of type Dst_V and an elementwise edge_op (not dot), and writes
+ *     arg[v][f] = the edge id (R9; the local CSR position inside a view) of the in-edge whose
+ *                 message supplied C[v][f]: the FIRST edge id attaining the extreme under the
+ *                 total order -0 < +0 (R12); -1 for zero in-degree rows (C = 0, R7).
+ *   arg: device int32 [V][F], row stride ld_arg >= F.  One kernel launch; deterministic.
+ *   Errors: as ug_op_run; UG_ERR_UNSUPPORTED_OP for sum/mean/assign or dot.
+ */
+ug_status ug_op_run_arg(const ug_graph *g, const ug_op_info *op, int32_t *arg, int64_t ld_arg,
+                        void *stream);
+
+/*
+ * ug_arg_scatter -- backward of a max/min aggregation through its arg capture:
+ *     for every v, f with e = arg[v][f] >= 0:  out[row(e)][f / (W / out_width)] += grad[v][f]
+ *   row(e) = src vertex of edge e (target_type UG_T_SRC_V: d/dA of copy_u_max) or e itself
+ *   (UG_T_EDGE: d/dA of copy_e_max).  out is ACCUMULATED into (zero it first); fp32 atomics,
+ *   so sums of several contributions to one element are order-dependent within rounding.
+ *   arg [V][W] (ld_arg), grad [V][W] (ld_grad), out [rows][out_width] (ld_out): device.
+ *   Errors: UG_ERR_INVALID_ARG, UG_ERR_UNSUPPORTED_OP (other target types), UG_ERR_SHAPE.
+ */
+ug_status ug_arg_scatter(const ug_graph *g, const int32_t *arg, int64_t ld_arg, int32_t W,
+                         const float *grad, int64_t ld_grad, int32_t target_type, float *out,
+                         int64_t ld_out, int32_t out_width, void *stream);
+
 /* Schedule <-> text, Table 9 notation ("TE_G1_T16", "SV_G2048_F64"). */
 ug_status ug_schedule_parse(const char *text, ug_schedule *out);
 ug_status ug_schedule_format(const ug_schedule *s, char *buf, size_t len);

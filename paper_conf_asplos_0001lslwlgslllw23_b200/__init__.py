@@ -20,7 +20,7 @@ from ._ffi import (EDGE_OPS, GATHER_OPS, STRATEGIES, TTYPES, UgError, UgOpInfo, 
                    UgTensor, check, lib)
 
 __all__ = ["Graph", "op_run", "prepare", "PreparedOp", "schedule_select", "launch_count", "parse_schedule",
-           "format_schedule", "validate", "edge_permute", "selector_load", "gat_attention", "UgError", "version"]
+           "format_schedule", "validate", "edge_permute", "selector_load", "gat_attention", "op_run_arg", "arg_scatter", "UgError", "version"]
 
 
 def version():
@@ -304,4 +304,32 @@ def gat_attention(graph, el, er, z, heads, slope=0.2, out=None, attn=None, strea
     pa, la = (None, 0) if attn is None else _mat(attn, "attn")
     check(lib.ug_gat_attention(graph.handle, pel, lel, per, ler, pz, lz, F, H, float(slope), po, lo, pa, la,
                                _current_stream(stream)), "ug_gat_attention")
+    return out
+
+
+def op_run_arg(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, C=None, F=None, H=None,
+               arg=None, stream=None):
+    """max/min aggregation with arg capture (ug_op_run_arg): fills C [V, F] as
+    op_run would and returns arg [V, F] int32 = the supplying edge id (first on ties, -1 for
+    zero in-degree rows)."""
+    import torch
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, "v", F, H)
+    if arg is None:
+        arg = torch.empty(C.shape[0], C.shape[1], dtype=torch.int32, device=C.device)
+    if arg.dtype != torch.int32 or arg.dim() != 2 or arg.stride(1) != 1:
+        raise TypeError("arg must be a 2-D int32 tensor with unit column stride")
+    check(lib.ug_op_run_arg(graph.handle, ctypes.byref(info), arg.data_ptr(), max(arg.stride(0), arg.shape[1]),
+                            _current_stream(stream)), "ug_op_run_arg")
+    return arg
+
+
+def arg_scatter(graph, arg, grad, target_type, out, stream=None):
+    """out[row(e)][f / (W / out_width)] += grad[v][f] for e = arg[v][f] >= 0 (ug_arg_scatter);
+    target_type "u" (row = src of e) or "e" (row = e)."""
+    W = int(arg.shape[1])
+    pg, lg = _mat(grad, "grad")
+    po, lo = _mat(out, "out")
+    check(lib.ug_arg_scatter(graph.handle, arg.data_ptr(), max(arg.stride(0), W), W, pg, lg, TTYPES[target_type],
+                             po, lo, int(out.shape[1] if out.dim() == 2 else 1), _current_stream(stream)),
+          "ug_arg_scatter")
     return out

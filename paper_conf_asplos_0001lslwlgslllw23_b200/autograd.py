@@ -10,14 +10,17 @@ the reversed graph.  Every backward step is again a graph operator of the 160-op
     hence the rows of w -- are unchanged)
   * d/dw of u_mul_e_sum(X, w)     = u_dot_v message creation over the forward graph:
     dw[e, h] = sum_{d in head h} X[src(e)][d] * dY[dst(e)][d]
-max / min backward (arg-max capture) is not provided.
+  * d/dX of copy_u_max / copy_u_min(X) and d/dE of copy_e_max / copy_e_min(E): the forward
+    records which in-edge supplied every output element (ug_op_run_arg; first edge id on
+    ties) and the backward scatters dY to that edge's source row (or to the edge itself)
+    with ug_arg_scatter
 """
 from __future__ import annotations
 
 import numpy as np
 import torch
 
-from . import Graph, op_run
+from . import Graph, arg_scatter, op_run, op_run_arg
 
 
 class GraphPair:
@@ -99,3 +102,38 @@ def u_mul_e_sum(gp: GraphPair, X, w):
     if w.dim() == 1:
         w = w.view(-1, 1)
     return _UMulESum.apply(gp, X, w)
+
+
+class _CopyExtreme(torch.autograd.Function):
+    @staticmethod
+    def forward(ctx, gp, X, a_type, gather):
+        F = X.shape[1]
+        Y = torch.empty(gp.V, F, device=X.device)
+        arg = op_run_arg(gp.fwd, "copy_lhs", gather, A=X.contiguous(), a_type=a_type, C=Y, F=F)
+        ctx.gp, ctx.a_type, ctx.rows = gp, a_type, X.shape[0]
+        ctx.save_for_backward(arg)
+        return Y
+
+    @staticmethod
+    def backward(ctx, dY):
+        (arg,) = ctx.saved_tensors
+        dX = torch.zeros(ctx.rows, dY.shape[1], device=dY.device)
+        arg_scatter(ctx.gp.fwd, arg, dY.contiguous(), ctx.a_type, dX)
+        return None, dX, None, None
+
+
+def copy_u_max(gp: GraphPair, X):
+    return _CopyExtreme.apply(gp, X, "u", "max")
+
+
+def copy_u_min(gp: GraphPair, X):
+    return _CopyExtreme.apply(gp, X, "u", "min")
+
+
+def copy_e_max(gp: GraphPair, Ee):
+    """Ee: [E, F] edge features in edge-id order."""
+    return _CopyExtreme.apply(gp, Ee, "e", "max")
+
+
+def copy_e_min(gp: GraphPair, Ee):
+    return _CopyExtreme.apply(gp, Ee, "e", "min")

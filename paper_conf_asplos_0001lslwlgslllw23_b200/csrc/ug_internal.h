@@ -93,6 +93,12 @@ struct GatArgs {
 cudaError_t launch_gat(const GraphArgs &g, const GatArgs &a, int vec, int L, const SplitPlan &plan,
                        const int32_t *slot_row, float *sacc, float *sst, int64_t sld, int64_t nfc,
                        int32_t *counters, cudaStream_t s);
+cudaError_t launch_argext(int kedge, int gather, const GraphArgs &g, const OpArgs &op, int L, const SplitPlan &plan,
+                          const int32_t *slot_row, float *sval, int32_t *sarg, int64_t sld, int32_t *counters,
+                          int32_t *arg, int64_t ld_arg, cudaStream_t s);
+cudaError_t launch_argscatter(const int32_t *arg, int64_t ld_arg, const float *grad, int64_t ld_grad, int64_t V, int W,
+                              bool to_src, const int32_t *col, const int32_t *src_of_eid, float *out, int64_t ld_out,
+                              int div, cudaStream_t s);
 cudaError_t launch_permute(const int32_t *eid, const float *in, float *out, int64_t E, int width,
                            cudaStream_t s);
 
@@ -134,5 +140,7 @@ struct ug_graph {
     // per-(split row, column tile) arrival counters of single-launch split-row merges
     // (ug_gat_attention), keyed by chunk size * 65536 + column tiles; zero between calls
     mutable std::map<int64_t, int32_t *> counters;
+    // src vertex by edge id (device), built on first use when eid is not the identity
+    mutable int32_t *d_src_of_eid = nullptr;
     mutable std::vector<void *> plan_allocs;
 };

@@ -523,3 +523,77 @@ extern "C" ug_status ug_gat_attention(const ug_graph *g, const float *el, int64_
     if (e != cudaSuccess) return set_error(UG_ERR_CUDA, std::string("ug_gat_attention: ") + cudaGetErrorString(e));
     return UG_OK;
 }
+
+// ------------------------------------------------------------------------- arg capture (f2)
+extern "C" ug_status ug_op_run_arg(const ug_graph *g, const ug_op_info *op, int32_t *arg, int64_t ld_arg,
+                                   void *stream) {
+    using namespace ug;
+    Lowered lw;
+    ug_status st = lower(g, op, &lw);
+    if (st != UG_OK) return st;
+    if (g->host_only) return set_error(UG_ERR_INVALID_ARG, "ug_op_run_arg needs a device graph");
+    if (lw.to_edges || lw.dot || (lw.gather != UG_GATHER_MAX && lw.gather != UG_GATHER_MIN))
+        return set_error(UG_ERR_UNSUPPORTED_OP, "ug_op_run_arg: max/min aggregation of an elementwise message only");
+    if (!arg && g->V > 0) return set_error(UG_ERR_INVALID_ARG, "ug_op_run_arg: NULL arg");
+    if (ld_arg < lw.args.W) return set_error(UG_ERR_SHAPE, "ug_op_run_arg: ld_arg < F");
+    if (g->V == 0) return UG_OK;
+    const int W = lw.args.W;
+    int L = 1;
+    while (L < 32 && L < W) L <<= 1;
+    const int n_tiles = (W + L - 1) / L;
+    const int G = 32;
+    const SplitPlan *plan = nullptr;
+    if ((st = get_plan(g, G, &plan)) != UG_OK) return st;
+    if (plan->n_chunks * n_tiles >= (int64_t)1 << 31)
+        return set_error(UG_ERR_SHAPE, "ug_op_run_arg: more than 2^31 (chunk, tile) units");
+    int32_t *counters = nullptr;
+    if ((st = get_counters(g, G, n_tiles, plan->n_split_rows, &counters)) != UG_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    const int64_t sld = (W + 3) / 4 * 4;
+    float *scratch = nullptr;
+    if (plan->n_split_chunks > 0) {
+        ensure_pool_retains();
+        if (cudaMallocAsync((void **)&scratch, (size_t)plan->n_split_chunks * sld * 8, s) != cudaSuccess)
+            return set_error(UG_ERR_OOM, "ug_op_run_arg: scratch allocation failed");
+    }
+    int32_t *sarg = scratch ? reinterpret_cast<int32_t *>(scratch + plan->n_split_chunks * sld) : nullptr;
+    cudaError_t e = launch_argext(lw.kedge, lw.gather, graph_args(g), lw.args, L, *plan, plan->d_slot_row, scratch,
+                                  sarg, sld, counters, arg, ld_arg, s);
+    if (scratch) cudaFreeAsync(scratch, s);
+    if (e != cudaSuccess) return set_error(UG_ERR_CUDA, std::string("ug_op_run_arg: ") + cudaGetErrorString(e));
+    return UG_OK;
+}
+
+extern "C" ug_status ug_arg_scatter(const ug_graph *g, const int32_t *arg, int64_t ld_arg, int32_t W,
+                                    const float *grad, int64_t ld_grad, int32_t target_type, float *out,
+                                    int64_t ld_out, int32_t out_width, void *stream) {
+    using namespace ug;
+    if (!g) return set_error(UG_ERR_INVALID_ARG, "ug_arg_scatter: NULL graph");
+    if (g->host_only) return set_error(UG_ERR_INVALID_ARG, "ug_arg_scatter needs a device graph");
+    if (target_type != UG_T_SRC_V && target_type != UG_T_EDGE)
+        return set_error(UG_ERR_UNSUPPORTED_OP, "ug_arg_scatter: target must be a Src_V or Edge tensor");
+    if (W <= 0 || out_width <= 0 || W % out_width != 0 || ld_arg < W || ld_grad < W || ld_out < out_width)
+        return set_error(UG_ERR_SHAPE, "ug_arg_scatter: need out_width | W and ld >= width");
+    if (g->V == 0) return UG_OK;
+    if (!arg || !grad || !out) return set_error(UG_ERR_INVALID_ARG, "ug_arg_scatter: NULL data");
+    const int32_t *src_of_eid = nullptr;
+    if (target_type == UG_T_SRC_V && g->d_eid) {
+        std::lock_guard<std::mutex> lock(g->mu);
+        if (!g->d_src_of_eid) {
+            std::vector<int32_t> h(g->E);
+            for (int64_t k = 0; k < g->E; ++k) h[g->h_eid[k]] = g->h_col[k];
+            void *d = nullptr;
+            if (cudaMalloc(&d, std::max<size_t>(16, h.size() * 4)) != cudaSuccess)
+                return set_error(UG_ERR_OOM, "ug_arg_scatter: allocation failed");
+            g->plan_allocs.push_back(d);
+            if (!h.empty() && cudaMemcpy(d, h.data(), h.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess)
+                return set_error(UG_ERR_CUDA, "ug_arg_scatter: upload failed");
+            g->d_src_of_eid = (int32_t *)d;
+        }
+        src_of_eid = g->d_src_of_eid;
+    }
+    cudaError_t e = launch_argscatter(arg, ld_arg, grad, ld_grad, g->V, W, target_type == UG_T_SRC_V, g->d_col,
+                                      src_of_eid, out, ld_out, W / out_width, (cudaStream_t)stream);
+    if (e != cudaSuccess) return set_error(UG_ERR_CUDA, std::string("ug_arg_scatter: ") + cudaGetErrorString(e));
+    return UG_OK;
+}
