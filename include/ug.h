@@ -181,6 +181,11 @@ ug_status ug_schedule_select(const ug_graph *g, const ug_op_info *op, ug_schedul
 /* Replace the selector table with the JSON file at `path` (format in DESIGN.md). */
 ug_status ug_selector_load(const char *path);
 
+/* Replace the learned selector model (tier 2 of ug_schedule_select) with the
+ * tree file at `path` (text format written by scripts/train_selector.py; default:
+ * selector_model.txt next to libugraph.so, or $UG_SELECTOR_MODEL).  "" unloads the model. */
+ug_status ug_selector_load_model(const char *path);
+
 /*
  * ug_op_run -- one unified-operator call (the paper's uGrapher(Graph_Tensor, op_info,
  * parallel_info)).  sched NULL or strategy UG_SCHED_AUTO -> ug_schedule_select.

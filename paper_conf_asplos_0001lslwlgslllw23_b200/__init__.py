@@ -20,7 +20,7 @@ from ._ffi import (EDGE_OPS, GATHER_OPS, STRATEGIES, TTYPES, UgError, UgOpInfo, 
                    UgTensor, check, lib)
 
 __all__ = ["Graph", "op_run", "prepare", "PreparedOp", "schedule_select", "launch_count", "parse_schedule",
-           "format_schedule", "validate", "edge_permute", "selector_load", "gat_attention", "op_run_arg", "arg_scatter", "UgError", "version"]
+           "format_schedule", "validate", "edge_permute", "selector_load", "selector_load_model", "gat_attention", "op_run_arg", "arg_scatter", "UgError", "version"]
 
 
 def version():
@@ -274,6 +274,11 @@ def edge_permute(graph, inp, out, stream=None):
 
 def selector_load(path):
     check(lib.ug_selector_load(str(path).encode()), "ug_selector_load")
+
+
+def selector_load_model(path):
+    """Load the learned selector trees (ug_selector_load_model); "" unloads them."""
+    check(lib.ug_selector_load_model(str(path).encode()), "ug_selector_load_model")
 
 
 def _mat(x, name):

@@ -63,6 +63,7 @@ SIGNATURES = {
     "ug_op_validate": ([_p, ctypes.POINTER(UgOpInfo)], _st),
     "ug_schedule_select": ([_p, ctypes.POINTER(UgOpInfo), ctypes.POINTER(UgSchedule)], _st),
     "ug_selector_load": ([ctypes.c_char_p], _st),
+    "ug_selector_load_model": ([ctypes.c_char_p], _st),
     "ug_op_run": ([_p, ctypes.POINTER(UgOpInfo), ctypes.POINTER(UgSchedule), _p], _st),
     "ug_op_run_events": ([_p, ctypes.POINTER(UgOpInfo), ctypes.POINTER(UgSchedule), _p, _p, _p], _st),
     "ug_op_launch_count": ([_p, ctypes.POINTER(UgOpInfo), ctypes.POINTER(UgSchedule),

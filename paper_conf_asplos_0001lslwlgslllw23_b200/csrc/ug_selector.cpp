@@ -1,15 +1,23 @@
 // ug_selector.cpp -- schedule selection when parallel_info is absent.
 //
-// The paper trains LightGBM on Table 7's features; this build replaces the
-// learned model by a table of schedules MEASURED on B200 (bench/sweep.py writes
-// selector_table.json), keyed by the Table 7 features plus the feature width F that Fig. 7
-// shows matters: op class, F, mean in-degree, degree CV (= std_nnz /
-// mean), V.  First matching entry wins; no match falls back to the priors below (Table 9's
-// observations, re-derived for B200 in DESIGN.md).  Lookup is a linear scan
-// over a few hundred entries: well under the paper's 0.2 ms budget.
+// The paper trains LightGBM on Table 7's features.  This build has three
+// tiers, consulted in order:
+//  1. a table of schedules MEASURED on B200 for the named configs (scripts/sweep.py writes
+//     selector_table.json), keyed by the Table 7 features plus the feature width F that Fig. 7
+//     shows matters: op class, F, mean in-degree, degree CV (= std_nnz /
+//     mean), V -- first matching entry wins;
+//  2. a learned model (selector_model.txt, scripts/train_selector.py): per op class a
+//     cost-sensitive regression tree trained on a synthetic B200 corpus of graphs
+//     (scripts/selector_corpus.py), features log2 V, log2 E, log2 mean degree, CV,
+//     log2(max degree / mean), log2 F; each leaf names the schedule with the lowest mean
+//     log-slowdown of its training points;
+//  3. priors (Table 9's observations, re-derived for B200 in DESIGN.md).
+// Each lookup is a linear scan / a tree walk of a few nodes: far under the paper's 0.2 ms
+// budget.
 #include <dlfcn.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cctype>
 #include <cstdlib>
 #include <cstring>
@@ -33,6 +41,16 @@ struct Entry {
 static std::mutex g_mu;
 static std::vector<Entry> g_table;
 static bool g_loaded = false;
+
+// Learned model: one tree per op class (index = class_of()).
+struct Node {
+    int feature = -1;       // -1: leaf
+    double thr = 0;
+    int left = -1, right = -1;
+    ug_schedule sched{};
+};
+static std::vector<Node> g_trees[6];
+static bool g_model_loaded = false;
 
 static int class_of(const std::string &s) {
     if (s == "msg") return 0;
@@ -126,6 +144,83 @@ static ug_status load_file(const std::string &path, bool quiet) {
     return UG_OK;
 }
 
+static std::string default_model_path() {
+    const char *env = std::getenv("UG_SELECTOR_MODEL");
+    if (env) return env;   // "" disables the model
+    std::string t = default_table_path();
+    size_t sl = t.rfind('/');
+    return (sl == std::string::npos ? std::string(".") : t.substr(0, sl)) + "/selector_model.txt";
+}
+
+// Text format of scripts/train_selector.py: "class <name> <n>" then n lines
+// "<id> <feature> <threshold> <left> <right> <schedule|->"; '#' lines are comments.
+static ug_status load_model(const std::string &path, bool quiet) {
+    std::ifstream in(path);
+    if (!in) return quiet ? UG_OK : set_error(UG_ERR_INVALID_ARG, "cannot open " + path);
+    std::vector<Node> trees[6];
+    std::string line;
+    int cls = -1, remaining = 0;
+    while (std::getline(in, line)) {
+        if (line.empty() || line[0] == '#') continue;
+        std::istringstream ls(line);
+        if (remaining == 0) {
+            std::string kw, name;
+            int n = 0;
+            if (!(ls >> kw >> name >> n) || kw != "class" || n <= 0)
+                return set_error(UG_ERR_INVALID_ARG, "selector model " + path + ": bad class line: " + line);
+            cls = class_of(name);
+            if (cls < 0) return set_error(UG_ERR_INVALID_ARG, "selector model: unknown class " + name);
+            trees[cls].assign(n, Node{});
+            remaining = n;
+            continue;
+        }
+        int id, f, l, r;
+        double thr;
+        std::string sched;
+        if (!(ls >> id >> f >> thr >> l >> r >> sched) || id < 0 || id >= (int)trees[cls].size())
+            return set_error(UG_ERR_INVALID_ARG, "selector model " + path + ": bad node line: " + line);
+        Node &nd = trees[cls][id];
+        nd.feature = f;
+        nd.thr = thr;
+        nd.left = l;
+        nd.right = r;
+        if (f < 0 && ug_schedule_parse(sched.c_str(), &nd.sched) != UG_OK)
+            return set_error(UG_ERR_INVALID_ARG, "selector model: bad schedule " + sched);
+        if (f >= 6 || (f >= 0 && (l < 0 || r < 0 || l >= (int)trees[cls].size() || r >= (int)trees[cls].size())))
+            return set_error(UG_ERR_INVALID_ARG, "selector model: bad node " + std::to_string(id));
+        --remaining;
+    }
+    if (remaining) return set_error(UG_ERR_INVALID_ARG, "selector model " + path + ": truncated");
+    for (int c = 0; c < 6; ++c) g_trees[c] = std::move(trees[c]);
+    return UG_OK;
+}
+
+static bool model_select(const ug_graph *g, const Lowered &lw, ug_schedule *out) {
+    const std::vector<Node> &t = g_trees[lw.op_class];
+    if (t.empty() || g->V <= 0 || g->E <= 0) return false;
+    const double mean = std::max(g->mean_deg, 1e-9);
+    const double x[6] = {std::log2((double)g->V), std::log2((double)g->E), std::log2(mean), g->std_nnz / mean,
+                         std::log2(std::max<double>(1.0, (double)g->max_deg) / mean), std::log2((double)lw.args.F)};
+    int n = 0;
+    for (int steps = 0; steps < 64 && t[n].feature >= 0; ++steps) n = x[t[n].feature] <= t[n].thr ? t[n].left : t[n].right;
+    if (t[n].feature >= 0) return false;
+    *out = t[n].sched;
+    return true;
+}
+
+// A measured schedule applied to this operator's layout: drop a forced vector width the
+// layout cannot take; an SV column tile may need more than 32 lanes at this layout's vector
+// width (measured with float4 rows, applied to float2 rows): keep 32 lanes.
+static ug_schedule adapt(const Lowered &lw, ug_schedule s) {
+    if (s.vec > lw.max_vec) s.vec = 0;
+    if (s.strategy == UG_SV && s.ftile > 0) {
+        const bool pack = (s.flags & UG_SCHED_PACK) && lw.pack_ok;
+        const int vec = std::max(1, std::min(pack ? 4 : lw.a_vec, lw.b_vec));
+        if (s.ftile / vec > 32 || s.ftile % vec) s.ftile = 32 * vec;
+    }
+    return s;
+}
+
 // Priors used when no measured entry matches.
 static ug_schedule prior(const ug_graph *g, const Lowered &lw) {
     ug_schedule s{};
@@ -160,9 +255,14 @@ ug_status select_schedule(const ug_graph *g, const Lowered &lw, ug_schedule *out
         g_loaded = true;
         load_file(default_table_path(), true);
     }
+    if (!g_model_loaded) {
+        g_model_loaded = true;
+        const std::string mp = default_model_path();
+        if (!mp.empty()) load_model(mp, true);
+    }
     const double F = lw.args.F, deg = g->mean_deg, V = (double)g->V;
     const double cv = g->mean_deg > 0 ? g->std_nnz / g->mean_deg : 0.0;
-    // exact class first, then the parent class (agg_bin / agg_ext -> agg)
+    // 1. measured table: exact class first, then the parent class (agg_bin / agg_ext -> agg)
     const int classes[2] = {lw.op_class, (lw.op_class == 4 || lw.op_class == 5) ? 1 : -2};
     for (int pass = 0; pass < 2; ++pass) {
         if (classes[pass] == -2) break;
@@ -171,19 +271,23 @@ ug_status select_schedule(const ug_graph *g, const Lowered &lw, ug_schedule *out
             if (F < e.F_lo || F > e.F_hi || deg < e.deg_lo || deg > e.deg_hi || cv < e.cv_lo || cv > e.cv_hi ||
                 V < e.V_lo || V > e.V_hi)
                 continue;
-            ug_schedule s = e.sched;
-            if (s.vec > lw.max_vec) s.vec = 0;   // table entry measured on an aligned layout
-            if (s.strategy == UG_SV && s.ftile > 0) {
-                // the entry's column tile may need more than 32 lanes at this layout's vector
-                // width (measured with float4 rows, applied to float2 rows): keep 32 lanes
-                const bool pack = (s.flags & UG_SCHED_PACK) && lw.pack_ok;
-                const int vec = std::max(1, std::min(pack ? 4 : lw.a_vec, lw.b_vec));
-                if (s.ftile / vec > 32 || s.ftile % vec) s.ftile = 32 * vec;
-            }
-            *out = s;
+            *out = adapt(lw, e.sched);
             return UG_OK;
         }
+        if (pass == 0) {
+            // 2. learned model of the exact class (only if its pick resolves on this layout)
+            ug_schedule s;
+            LaunchCfg cfg;
+            if (model_select(g, lw, &s)) {
+                s = adapt(lw, s);
+                if (resolve(g, lw, s, &cfg) == UG_OK) {
+                    *out = s;
+                    return UG_OK;
+                }
+            }
+        }
     }
+    // 3. priors
     *out = prior(g, lw);
     return UG_OK;
 }
@@ -196,6 +300,17 @@ extern "C" ug_status ug_schedule_select(const ug_graph *g, const ug_op_info *op,
     ug_status st = ug::lower(g, op, &lw);
     if (st != UG_OK) return st;
     return ug::select_schedule(g, lw, out);
+}
+
+extern "C" ug_status ug_selector_load_model(const char *path) {
+    if (!path) return ug::set_error(UG_ERR_INVALID_ARG, "NULL path");
+    std::lock_guard<std::mutex> lock(ug::g_mu);
+    ug::g_model_loaded = true;
+    if (!*path) {                       // "" unloads the model
+        for (auto &t : ug::g_trees) t.clear();
+        return UG_OK;
+    }
+    return ug::load_model(path, false);
 }
 
 extern "C" ug_status ug_selector_load(const char *path) {
