@@ -168,6 +168,25 @@ ug_status ug_graph_partition(const ug_graph *g, int32_t parts, int64_t *row_spli
  */
 ug_status ug_graph_view_rows(const ug_graph *g, int64_t r0, int64_t r1, ug_graph **view);
 
+/*
+ * ug_graph_reorder -- vertex renumbering for locality (node renumbering as
+ * orthogonal preprocessing).  Host only.  Writes perm[new_id] = old_id
+ * (host int32 [V]) for a whole square graph (not a view):
+ *   UG_ORDER_DEGREE: descending total (in + out) degree, ties by id;
+ *   UG_ORDER_RCM:    reverse Cuthill-McKee on the symmetrised graph.
+ * The caller renumbers its COO (src' = inv[src], dst' = inv[dst], edge ids unchanged),
+ * builds a new graph and gathers vertex tensors with ug_rows_gather(X, perm) -- results then
+ * come back in the new numbering (gather them with the inverse permutation).
+ */
+#define UG_ORDER_DEGREE 1
+#define UG_ORDER_RCM 2
+ug_status ug_graph_reorder(const ug_graph *g, int32_t method, int32_t *perm);
+
+/* out[i][0..width) = in[idx[i]][0..width) for i < rows (device pointers, row strides ld_in /
+ * ld_out >= width; idx device int32).  Asynchronous on `stream`. */
+ug_status ug_rows_gather(const float *in, int64_t ld_in, const int32_t *idx, int64_t rows, int32_t width,
+                         float *out, int64_t ld_out, void *stream);
+
 /* Validate op_info against the supported op set and shapes without running (host only). */
 ug_status ug_op_validate(const ug_graph *g, const ug_op_info *op);
 

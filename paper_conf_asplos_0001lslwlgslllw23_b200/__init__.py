@@ -20,7 +20,8 @@ from ._ffi import (EDGE_OPS, GATHER_OPS, STRATEGIES, TTYPES, UgError, UgOpInfo, 
                    UgTensor, check, lib)
 
 __all__ = ["Graph", "op_run", "prepare", "PreparedOp", "schedule_select", "launch_count", "parse_schedule",
-           "format_schedule", "validate", "edge_permute", "selector_load", "selector_load_model", "gat_attention", "op_run_arg", "arg_scatter", "UgError", "version"]
+           "format_schedule", "validate", "edge_permute", "selector_load", "selector_load_model", "gat_attention", "op_run_arg", "arg_scatter", "reorder", "rows_gather", "Renumbered", "UgError",
+           "version"]
 
 
 def version():
@@ -338,3 +339,59 @@ def arg_scatter(graph, arg, grad, target_type, out, stream=None):
                              po, lo, int(out.shape[1] if out.dim() == 2 else 1), _current_stream(stream)),
           "ug_arg_scatter")
     return out
+
+
+ORDERS = {"degree": 1, "rcm": 2}
+
+
+def reorder(graph, method="rcm"):
+    """perm[new_id] = old_id (ug_graph_reorder: "degree" or "rcm")."""
+    V = graph.stats()["V"]
+    perm = np.zeros(max(V, 1), np.int32)
+    check(lib.ug_graph_reorder(graph.handle, ORDERS[method], perm.ctypes.data), "ug_graph_reorder")
+    return perm[:V]
+
+
+def rows_gather(X, idx, out=None, stream=None):
+    """out[i] = X[idx[i]] on the device (ug_rows_gather); idx: int32 CUDA tensor."""
+    import torch
+    if out is None:
+        out = torch.empty(idx.shape[0], X.shape[1], device=X.device, dtype=X.dtype)
+    px, lx = _mat(X, "X")
+    po, lo = _mat(out, "out")
+    if idx.dtype != torch.int32 or not idx.is_cuda:
+        raise TypeError("idx must be an int32 CUDA tensor")
+    check(lib.ug_rows_gather(px, lx, idx.data_ptr(), int(idx.shape[0]), int(X.shape[1]), po, lo,
+                             _current_stream(stream)), "ug_rows_gather")
+    return out
+
+
+class Renumbered:
+    """A graph renumbered for locality: `graph` is built on the new ids; to_new(X) / to_old(Y)
+    move vertex tensors between numberings on the device.  Edge ids are unchanged."""
+
+    def __init__(self, num_vertices, src, dst, method="rcm"):
+        import torch
+        src = np.ascontiguousarray(src, np.int32)
+        dst = np.ascontiguousarray(dst, np.int32)
+        base = Graph(num_vertices, src, dst, host_only=True)
+        self.perm = reorder(base, method)
+        self.inv = np.empty_like(self.perm)
+        self.inv[self.perm] = np.arange(len(self.perm), dtype=np.int32)
+        nsrc, ndst = self.inv[src], self.inv[dst]
+        order = np.argsort(ndst, kind="stable")          # dst-sorted: identity edge positions
+        self.edge_order = order.astype(np.int32)         # new CSR position -> original edge id
+        self.graph = Graph(num_vertices, nsrc[order], ndst[order])
+        self._perm_d = torch.from_numpy(self.perm).cuda()
+        self._inv_d = torch.from_numpy(self.inv).cuda()
+        self._eord_d = torch.from_numpy(self.edge_order).cuda()
+
+    def to_new(self, X):
+        return rows_gather(X, self._perm_d)
+
+    def to_old(self, Y):
+        return rows_gather(Y, self._inv_d)
+
+    def edges_to_new(self, W):
+        """Edge tensor in original edge-id order -> the renumbered graph's edge order."""
+        return rows_gather(W, self._eord_d)

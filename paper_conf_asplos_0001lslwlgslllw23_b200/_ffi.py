@@ -73,6 +73,8 @@ SIGNATURES = {
                          _st),
     "ug_op_run_arg": ([_p, ctypes.POINTER(UgOpInfo), _p, _i64, _p], _st),
     "ug_arg_scatter": ([_p, _p, _i64, _i32, _p, _i64, _i32, _p, _i64, _i32, _p], _st),
+    "ug_graph_reorder": ([_p, _i32, _p], _st),
+    "ug_rows_gather": ([_p, _i64, _p, _i64, _i32, _p, _i64, _p], _st),
     "ug_schedule_parse": ([ctypes.c_char_p, ctypes.POINTER(UgSchedule)], _st),
     "ug_schedule_format": ([ctypes.POINTER(UgSchedule), ctypes.c_char_p, ctypes.c_size_t], _st),
     "ug_status_string": ([_st], ctypes.c_char_p),

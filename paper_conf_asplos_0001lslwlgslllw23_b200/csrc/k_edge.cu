@@ -250,3 +250,23 @@ cudaError_t launch_permute(const int32_t *eid, const float *in, float *out, int6
 }
 
 }  // namespace ug
+
+namespace ug {
+// out[i][:] = in[idx[i]][:] (vertex renumbering, ug_rows_gather): one warp per row, lanes
+// over the features.
+__global__ void k_rows_gather(const float *__restrict__ in, int64_t ld_in, const int32_t *__restrict__ idx,
+                              int64_t rows, int width, float *__restrict__ out, int64_t ld_out) {
+    const int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (w >= rows) return;
+    const float *src = in + (int64_t)idx[w] * ld_in;
+    float *dst = out + w * ld_out;
+    for (int f = lane; f < width; f += 32) dst[f] = __ldg(src + f);
+}
+
+cudaError_t launch_rows_gather(const float *in, int64_t ld_in, const int32_t *idx, int64_t rows, int width,
+                               float *out, int64_t ld_out, cudaStream_t s) {
+    k_rows_gather<<<(unsigned)cdiv(rows * 32, 256), 256, 0, s>>>(in, ld_in, idx, rows, width, out, ld_out);
+    return cudaGetLastError();
+}
+}  // namespace ug

@@ -110,14 +110,26 @@ __device__ __forceinline__ void gat_walk(const GraphArgs &g, const GatArgs &a, i
     }
 }
 
-// Attention output of edges k0 .. k1 of row v (the writer lane of each head).
+// Attention output of edges k0 + j, k0 + j + nh, ... < k1 of row v: the nh lanes of a head
+// split the edges, 4 independent loads in flight per lane.
 __device__ __forceinline__ void gat_attn(const GraphArgs &g, const GatArgs &a, int64_t k0, int64_t k1, int h,
-                                         float erv, float m, float den) {
-    for (int64_t k = k0; k < k1; ++k) {
-        const int64_t u = g.col[k];
-        const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
-        const float p = ex2(__fsub_rn(score2(__ldg(a.el + u * a.ld_el + h), erv, a.slope), m));
-        a.attn[e * a.ld_attn + h] = __fdiv_rn(p, den);
+                                         float erv, float m, float den, int j, int nh) {
+    constexpr int U = 4;
+    for (int64_t k = k0 + j; k < k1; k += (int64_t)U * nh) {
+        int64_t e[U];
+        float t[U];
+#pragma unroll
+        for (int q = 0; q < U; ++q) {
+            const int64_t kk = k + (int64_t)q * nh;
+            const int64_t kc = kk < k1 ? kk : k;
+            const int64_t u = g.col[kc];
+            e[q] = kk < k1 ? (g.eid ? (int64_t)g.eid[kc] : kc) : -1;
+            t[q] = __ldg(a.el + u * a.ld_el + h);
+        }
+#pragma unroll
+        for (int q = 0; q < U; ++q)
+            if (e[q] >= 0)
+                a.attn[e[q] * a.ld_attn + h] = __fdiv_rn(ex2(__fsub_rn(score2(t[q], erv, a.slope), m)), den);
     }
 }
 
@@ -161,7 +173,7 @@ __global__ void __launch_bounds__(256) k_gat(GraphArgs g, GatArgs a, int L_log2,
     if (ch.w < 0) {                                   // the row is one chunk: finalise here
         if (active) gat_store<VEC>(a, v, f, st, ch.z == ch.y);
         if constexpr (ATTN) {
-            if (active && (f - h * a.D) < VEC) gat_attn(g, a, ch.y, ch.z, h, erv, st.m, st.den);
+            if (active) gat_attn(g, a, ch.y, ch.z, h, erv, st.m, st.den, (f - h * a.D) / VEC, (a.D + VEC - 1) / VEC);
         }
         return;
     }
@@ -195,9 +207,9 @@ __global__ void __launch_bounds__(256) k_gat(GraphArgs g, GatArgs a, int L_log2,
     }
     if (active) gat_store<VEC>(a, v, f, st, false);
     if constexpr (ATTN) {
-        if (active && (f - h * a.D) < VEC) {
+        if (active) {
             const int64_t r0 = (int64_t)g.row_ptr[v] - g.rp_base, r1 = (int64_t)g.row_ptr[v + 1] - g.rp_base;
-            gat_attn(g, a, r0, r1, h, erv, st.m, st.den);
+            gat_attn(g, a, r0, r1, h, erv, st.m, st.den, (f - h * a.D) / VEC, (a.D + VEC - 1) / VEC);
         }
     }
 }

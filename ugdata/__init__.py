@@ -154,3 +154,23 @@ def values(rows, width, seed, tag, mode="float", role="num", k=8):
         x[z] = rng.uniform(-1.0, 1.0, int(z.sum())).astype(np.float32)
         z = x == 0.0
     return x
+
+
+def community_graph(V, E, blocks, p_in, seed, shuffle=True):
+    """Stochastic-block-style COO (no method arithmetic): vertex v belongs to block
+    v * blocks // V; each edge picks a destination uniformly and, with probability p_in, a
+    source in the same block (else anywhere).  Ids are then randomly relabelled (shuffle),
+    hiding the locality a renumbering (ug_graph_reorder) can recover.  Returned dst-sorted."""
+    rng = np.random.default_rng(seed)
+    dst = rng.integers(0, V, E).astype(np.int64)
+    blk = dst * blocks // V
+    lo = (blk * V + blocks - 1) // blocks
+    hi = ((blk + 1) * V + blocks - 1) // blocks
+    local = lo + (rng.random(E) * (hi - lo)).astype(np.int64)
+    anywhere = rng.integers(0, V, E)
+    src = np.where(rng.random(E) < p_in, local, anywhere)
+    if shuffle:
+        relabel = rng.permutation(V)
+        src, dst = relabel[src], relabel[dst]
+    order = np.argsort(dst, kind="stable")
+    return src[order].astype(np.int32), dst[order].astype(np.int32)
