@@ -173,13 +173,16 @@ ug_status ug_graph_view_rows(const ug_graph *g, int64_t r0, int64_t r1, ug_graph
  * orthogonal preprocessing).  Host only.  Writes perm[new_id] = old_id
  * (host int32 [V]) for a whole square graph (not a view):
  *   UG_ORDER_DEGREE: descending total (in + out) degree, ties by id;
- *   UG_ORDER_RCM:    reverse Cuthill-McKee on the symmetrised graph.
+ *   UG_ORDER_RCM:    reverse Cuthill-McKee on the symmetrised graph;
+ *   UG_ORDER_COMMUNITY: Rabbit-style community order (label propagation on the symmetrised
+ *                    graph, vertices grouped by community, descending degree inside).
  * The caller renumbers its COO (src' = inv[src], dst' = inv[dst], edge ids unchanged),
  * builds a new graph and gathers vertex tensors with ug_rows_gather(X, perm) -- results then
  * come back in the new numbering (gather them with the inverse permutation).
  */
 #define UG_ORDER_DEGREE 1
 #define UG_ORDER_RCM 2
+#define UG_ORDER_COMMUNITY 3
 ug_status ug_graph_reorder(const ug_graph *g, int32_t method, int32_t *perm);
 
 /* out[i][0..width) = in[idx[i]][0..width) for i < rows (device pointers, row strides ld_in /

@@ -341,11 +341,11 @@ def arg_scatter(graph, arg, grad, target_type, out, stream=None):
     return out
 
 
-ORDERS = {"degree": 1, "rcm": 2}
+ORDERS = {"degree": 1, "rcm": 2, "community": 3}
 
 
 def reorder(graph, method="rcm"):
-    """perm[new_id] = old_id (ug_graph_reorder: "degree" or "rcm")."""
+    """perm[new_id] = old_id (ug_graph_reorder: "degree", "rcm" or "community")."""
     V = graph.stats()["V"]
     perm = np.zeros(max(V, 1), np.int32)
     check(lib.ug_graph_reorder(graph.handle, ORDERS[method], perm.ctypes.data), "ug_graph_reorder")

@@ -14,7 +14,7 @@ pytestmark = pytest.mark.gpu
 ug = pytest.importorskip("paper_conf_asplos_0001lslwlgslllw23_b200")
 
 
-@pytest.mark.parametrize("method", ["rcm", "degree"])
+@pytest.mark.parametrize("method", ["rcm", "degree", "community"])
 @pytest.mark.parametrize("graph", ["multigraph", "community"])
 def test_renumbered_ops_match_oracle(method, graph):
     if graph == "multigraph":

@@ -19,7 +19,7 @@ def _shuffled(V, src, dst, seed):
     return r[src], r[dst]
 
 
-@pytest.mark.parametrize("method", ["degree", "rcm"])
+@pytest.mark.parametrize("method", ["degree", "rcm", "community"])
 def test_reorder_is_a_permutation(method):
     V = 500
     src, dst = ugdata.random_multigraph(V, 3000, 3)
@@ -68,3 +68,21 @@ def test_reorder_rejects_views():
     g = ug.Graph(V, src, dst, host_only=True)
     with pytest.raises(ug.UgError):
         ug.reorder(g.view_rows(0, 10), "rcm")
+
+
+def test_community_order_recovers_blocks():
+    """Block graph (200 blocks of 100 vertices, 90 % of edges inside a block) under random ids:
+    after the community order at least 85 % of the edges join vertices < 100 ids apart (all
+    intra-block edges, when each block becomes one id range); the shuffled ids have ~0.5 %."""
+    V, blocks = 20000, 200
+    src, dst = ugdata.community_graph(V, 300000, blocks, 0.9, 3)
+    g = ug.Graph(V, src, dst, host_only=True)
+    near = lambda p: _near(p, src, dst, V // blocks)
+    assert near(np.arange(V, dtype=np.int32)) < 0.02
+    assert near(ug.reorder(g, "community")) > 0.85
+
+
+def _near(perm, src, dst, width):
+    inv = np.empty_like(perm)
+    inv[perm] = np.arange(len(perm))
+    return float((np.abs(inv[src].astype(np.int64) - inv[dst]) < width).mean())
