@@ -22,6 +22,12 @@ KEYS = [
     "lts__t_sectors_srcunit_tex_op_read.sum",
     "lts__t_sector_hit_rate.pct",
     "lts__throughput.avg.pct_of_peak_sustained_elapsed",
+    "lts__throughput.max.pct_of_peak_sustained_elapsed",
+    "lts__lts2xbar_cycles_active.avg.pct_of_peak_sustained_elapsed",
+    "lts__lts2xbar_cycles_active.max.pct_of_peak_sustained_elapsed",
+    "lts__t_sectors_srcunit_tex.avg.pct_of_peak_sustained_elapsed",
+    "lts__t_sectors_srcunit_ltcfabric.sum",
+    "l1tex__m_xbar2l1tex_read_bytes.sum.pct_of_peak_sustained_elapsed",
     "l1tex__t_bytes.sum",
     "l1tex__t_sector_hit_rate.pct",
     "sm__throughput.avg.pct_of_peak_sustained_elapsed",

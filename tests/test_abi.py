@@ -226,6 +226,7 @@ def test_selector_table_load_and_match(tmp_path):
                  '  "V_lo": 1000, "V_hi": 10000, "schedule": "BV_G4_B256"},\n'
                  ' {"class": "msg", "F_lo": 8, "F_hi": 20, "schedule": "WE_G16_T1"}]}')
     ug.selector_load(t)
+    ug.selector_load_model("")          # tier 2 off: a table miss goes straight to the priors
     X, Y = torch.zeros(V, 16), torch.zeros(V, 16)
     assert ug.schedule_select(g, "copy_lhs", "sum", A=X, a_type="u", C=Y, c_type="v") == "BV_G4_B256"
     Z = torch.zeros(E, 16)
@@ -236,7 +237,10 @@ def test_selector_table_load_and_match(tmp_path):
     bad.write_text('{"entries": [{"class": "agg", "schedule": "XX_G1"}]}')
     with pytest.raises(ug.UgError):
         ug.selector_load(bad)
-    # restore the shipped table (if any) for later tests
+    # restore the shipped table and model (if any) for later tests
+    model = os.path.join(ROOT, "paper_conf_asplos_0001lslwlgslllw23_b200", "selector_model.txt")
+    if os.path.exists(model):
+        ug.selector_load_model(model)
     shipped = os.path.join(ROOT, "paper_conf_asplos_0001lslwlgslllw23_b200", "selector_table.json")
     if os.path.exists(shipped):
         ug.selector_load(shipped)
