@@ -25,10 +25,10 @@ namespace ug {
 // / full width, 4 / 5 B is Src_V with broadcast / full width.  All offsets are 32-bit (the
 // host checks rows * ld < 2^32).  The last, partial group of UF edges is predicated (its
 // missing slots re-read the row's last edge, an L1 hit, and are not combined), so short rows
-// never fall into a serial one-edge-at-a-time tail.  Advances k to k1.
+// never fall into a serial one-edge-at-a-time tail.  
 template <int KE, int GOP, int VEC, int BM>
-__device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t &k,
-                                                int64_t k1, int f, int64_t cb, float (&acc)[VEC]) {
+__device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t k,
+                                                const int64_t k1, int f, int64_t cb, float (&acc)[VEC]) {
     // row gathers in flight per lane: 16 (measured +3 % over 8 on C5 at VEC 2), 8 for float4 rows;
     // half that when a B operand is loaded per edge (register budget of 40 for 6 CTAs / SM)
 #ifndef UG_BM2_UF
@@ -87,7 +87,6 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
     // the last, partial group: predicated half-groups (fewer registers), not a serial tail
     constexpr int UH = UF / 2 > 0 ? UF / 2 : 1;
     for (; k < k1; k += UH) group(std::true_type{}, std::integral_constant<int, UH>{});
-    k = k1;
 }
 
 // BM < 0: generic addressing (any operand types, eid); BM >= 0: the fast path with the B
@@ -105,7 +104,9 @@ __global__ void __launch_bounds__(256, (BM == 0) ? 8 : (BM == 2 ? UG_BM2_MINB : 
     const int lane = (int)(t & ((1 << L_log2) - 1));
     const int64_t u = t >> L_log2;
     if (u >= n_chunks * n_tiles) return;
-    const int tile = (int)(u / n_chunks);
+    // unit -> (column tile, chunk): no division for one tile, a 32-bit one below 2^31 units
+    int tile = 0;
+    if (n_tiles > 1) tile = u < INT32_MAX ? (int)((uint32_t)u / (uint32_t)n_chunks) : (int)(u / n_chunks);
     const int64_t c = u - (int64_t)tile * n_chunks;
     const int f = tile * ftile + lane * VEC;
     if (f >= op.W) return;
@@ -134,6 +135,7 @@ __global__ void __launch_bounds__(256, (BM == 0) ? 8 : (BM == 2 ? UG_BM2_MINB : 
             // column index, so each in-edge costs ~6 instructions per lane.  The B operand's
             // addressing mode BM is a template parameter (a Dst_V operand is loaded once).
             split_fast_loop<KE, GOP, VEC, BM>(g, op, v, k, k1, f, cb, acc);
+            k = k1;
         } else {
             for (; k + U <= k1; k += U) {
                 float m[U][VEC];
@@ -160,7 +162,8 @@ __global__ void __launch_bounds__(256, (BM == 0) ? 8 : (BM == 2 ? UG_BM2_MINB : 
         // outputs are written once: evict_first keeps them from displacing the X slab in L2
         const uint64_t wpol = l2_policy_evict_first();
         if (ch.w < 0) {
-            const int64_t deg = (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
+            // sum needs no degree (an empty row's accumulator is already +0)
+            const int64_t deg = GOP == UG_GATHER_SUM ? 1 : (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
             float out[VEC];
 #pragma unroll
             for (int i = 0; i < VEC; ++i) out[i] = g_finalize<GOP>(acc[i], deg);

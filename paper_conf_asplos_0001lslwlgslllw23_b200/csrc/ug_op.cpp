@@ -210,6 +210,24 @@ static ug_status get_plan(const ug_graph *g, int G, const SplitPlan **out) {
             }
         }
     }
+    // Longest chunks first (stable): the lane groups sharing a warp then walk equally long
+    // in-edge lists (no lanes idling while the warp's longest row finishes -- with CV ~1.8 the
+    // longest of 4 rows is far above their mean), and the longest units start first (LPT
+    // balance over the SMs).  Kernels address partials by scratch slot, never by chunk
+    // position, so the order is free.  UG_SV_ORDER=row keeps row order (A/B measurements).
+    const char *order = std::getenv("UG_SV_ORDER");
+    if (!(order && std::string(order) == "row")) {
+        const size_t nc = chunks.size() / 4;
+        std::vector<int32_t> idx(nc);
+        for (size_t i = 0; i < nc; ++i) idx[i] = (int32_t)i;
+        std::stable_sort(idx.begin(), idx.end(), [&](int32_t a, int32_t b) {
+            return chunks[4 * a + 2] - chunks[4 * a + 1] > chunks[4 * b + 2] - chunks[4 * b + 1];
+        });
+        std::vector<int32_t> sorted(chunks.size());
+        for (size_t i = 0; i < nc; ++i)
+            for (int j = 0; j < 4; ++j) sorted[4 * i + j] = chunks[4 * (size_t)idx[i] + j];
+        chunks.swap(sorted);
+    }
     SplitPlan p;
     p.n_chunks = (int64_t)chunks.size() / 4;
     p.n_split_rows = (int64_t)split.size() / 4;

@@ -49,6 +49,8 @@ def main():
             elif mode == "flush":
                 junk.fill_(float(i))
             k0, k1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            k0.record(s)    # materialise the cudaEvent_t handles ug_op_run_events records into
+            k1.record(s)
             s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             s0.record(s)
             ug.op_run_events(g, "copy_lhs", "sum", k0, k1, A=A, a_type="u", C=C, c_type="v", schedule=sched)

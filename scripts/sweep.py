@@ -61,7 +61,7 @@ def candidates(cls, F, E, quick=False):
         c += [f"BE_G{g}" for g in (64, 512)]
         if cls != "dot_agg":
             fts = [f for f in (16, 32, 64, 128) if f <= max(16, 2 * F)]
-            c += [f"SV_G{g}_F{f}" for g in (16, 32, 128, 512, 2048) for f in fts]
+            c += [f"SV_G{g}_F{f}" for g in (16, 32, 64, 128, 512, 2048) for f in fts]
             c += [f"SV_G{g}_F{f}_P1" for g in (32, 128, 512) for f in (64, 128) if f <= max(16, 2 * F)]
         else:
             c += [f"SV_G{g}" for g in (256, 1024)]
