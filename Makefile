@@ -7,7 +7,7 @@ BUILD   := build
 LIB     := $(PKG)/libugraph.so
 ARCH    := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -prec-div=true -prec-sqrt=true -fmad=true \
-           -Iinclude -I$(SRC) -Xptxas -v
+           -Iinclude -I$(SRC) -Xptxas -v $(EXTRA)
 CU      := $(wildcard $(SRC)/*.cu)
 CPP     := $(wildcard $(SRC)/*.cpp)
 OBJ     := $(patsubst $(SRC)/%.cu,$(BUILD)/%.o,$(CU)) $(patsubst $(SRC)/%.cpp,$(BUILD)/%.o,$(CPP))
