@@ -174,43 +174,18 @@ __device__ __forceinline__ int unit_tile(int64_t u, int64_t n_chunks, int n_tile
     return u < INT32_MAX ? (int)((uint32_t)u / (uint32_t)n_chunks) : (int)(u / n_chunks);
 }
 
-#ifndef UG_SV_PERSIST
-#define UG_SV_PERSIST 0
-#endif
-
-// UG_SV_PERSIST: one resident wave of CTAs; each lane group walks units u, u + S, ... (S =
-// lane groups in the grid) and loads the next unit's chunk descriptor before working on the
-// current one, taking the descriptor load off the per-unit dependency chain.
 template <int KE, int GOP, int VEC, int BM>
 __global__ void __launch_bounds__(256, (BM == 0) ? UG_BM0_MINB : (BM == 2 ? UG_BM2_MINB : (BM > 0 ? (VEC == 4 ? 5 : 6) : 4))) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
                                                int64_t n_chunks, int L_log2, int ftile, int n_tiles,
                                                float *__restrict__ scratch, int64_t sld) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int lane = (int)(t & ((1 << L_log2) - 1));
-    const int64_t n_units = n_chunks * n_tiles;
-    int64_t u = t >> L_log2;
-    if (u >= n_units) return;
-#if UG_SV_PERSIST
-    const int64_t stride = ((int64_t)gridDim.x * blockDim.x) >> L_log2;
-    int tile = unit_tile(u, n_chunks, n_tiles);
-    int4 ch = chunks[u - (int64_t)tile * n_chunks];
-    for (;;) {
-        const int64_t un = u + stride;
-        const int tn = un < n_units ? unit_tile(un, n_chunks, n_tiles) : tile;
-        const int4 chn = un < n_units ? chunks[un - (int64_t)tn * n_chunks] : ch;
-        const int f = tile * ftile + lane * VEC;
-        if (f < op.W) split_unit<KE, GOP, VEC, BM>(g, op, ch, f, scratch, sld);
-        if (un >= n_units) break;
-        u = un;
-        tile = tn;
-        ch = chn;
-    }
-#else
+    const int64_t u = t >> L_log2;
+    if (u >= n_chunks * n_tiles) return;
     const int tile = unit_tile(u, n_chunks, n_tiles);
     const int f = tile * ftile + lane * VEC;
     if (f >= op.W) return;
     split_unit<KE, GOP, VEC, BM>(g, op, chunks[u - (int64_t)tile * n_chunks], f, scratch, sld);
-#endif
 }
 
 // Fix-up of split rows: combine the row's partials in chunk order, finalise, store.
@@ -237,17 +212,6 @@ __global__ void k_split_fix(GraphArgs g, OpArgs op, const int4 *__restrict__ spl
 #pragma unroll
     for (int i = 0; i < VEC; ++i) acc[i] = g_finalize<GOP>(acc[i], deg);
     st_out<VEC>(op.C + v * op.c_ld + f, acc, op.W - f, op.c_vec);
-}
-
-// SMs of the current device (cached; the node's GPUs are identical B200s).
-static inline int sm_count() {
-    static int n = 0;
-    if (n == 0) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
-    }
-    return n;
 }
 
 // Launch of one edge_op's SV instances (explicitly instantiated per KE in k_split*.cu).
@@ -277,17 +241,8 @@ cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, co
     const int bm = !fast ? -1 : KE == K_COPY ? 0
                  : op.B.type == UG_T_DST_V ? 1 : (op.B.type == UG_T_EDGE ? 2 + bfl : 4 + bfl);
 #define UG_SV_LAUNCH(BMV)                                                                               \
-    do {                                                                                                \
-        int64_t gr = grid;                                                                              \
-        if (UG_SV_PERSIST) {                                                                            \
-            static int occ = 0;                                                                         \
-            if (occ == 0) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_split<KE, GOP, VEC, BMV>, \
-                                                                        c.block, 0);                    \
-            gr = std::min<int64_t>(grid, (int64_t)std::max(1, occ) * sm_count());                       \
-        }                                                                                               \
-        k_split<KE, GOP, VEC, BMV><<<(unsigned)gr, c.block, 0, s>>>(g, op, chunks, plan.n_chunks, L_log2, \
-                                                                     c.ftile, n_tiles, scratch, sld);   \
-    } while (0)
+    k_split<KE, GOP, VEC, BMV><<<(unsigned)grid, c.block, 0, s>>>(g, op, chunks, plan.n_chunks, L_log2, \
+                                                                 c.ftile, n_tiles, scratch, sld)
     UG_DISPATCH_VEC(c.vec, VEC,
         UG_DISPATCH_GOP(gather, GOP, {
             if constexpr (GOP == UG_GATHER_ASSIGN) {
