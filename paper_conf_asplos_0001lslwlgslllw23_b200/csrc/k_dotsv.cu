@@ -1,0 +1,175 @@
+// k_dotsv.cu -- `dot` between a Src_V and a Dst_V operand (u_dot_v / v_dot_u, the SDDMM of
+// config C4; reading R5) under the SV schedule: the Dst_V row is loaded ONCE per work unit
+// and kept in registers, so each in-edge gathers only the source row (half the L2->SM bytes
+// of the edge-unit kernel, which loads both rows per edge).
+//
+// Work unit = one SV chunk (row v, in-edges [k0, k1), scratch slot; longest first, see
+// get_plan).  L lanes serve a unit, in aligned groups of w = D/(NJ*VEC) lanes per head: lane
+// (o, l) of head o owns the VEC-wide feature chunks o*D + (j*w + l)*VEC, j < NJ, so every load
+// instruction of a group reads w*VEC contiguous floats of the head (one 128-byte line per 8
+// lanes at VEC 4).  A head's message is an in-register FFMA chain over the lane's NJ*VEC
+// features, then a log2(w)-step xor butterfly inside the group.  UE in-edges are gathered per
+// step (16 floats per lane in flight), their column indices loaded first.  Message creation
+// (C = Edge) stores one value per (edge, head); reductions keep the running value in the
+// group's lanes and finalise owned rows in registers, split rows through the SV scratch and
+// k_split_fix (chunk order, deterministic).
+#include "k_split.cuh"
+
+namespace ug {
+
+template <int GOP, int VEC, int NJ>
+__global__ void __launch_bounds__(256, 4) k_dotsv(GraphArgs g, OpArgs op, bool a_is_src, const int4 *__restrict__ chunks,
+                                                  int64_t n_chunks, int L_log2, int w_log2,
+                                                  float *__restrict__ scratch, int64_t sld) {
+    constexpr int UE = NJ * VEC >= 16 ? 1 : 16 / (NJ * VEC);   // in-edges per step
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int L = 1 << L_log2, w = 1 << w_log2;
+    const int lane = (int)(t & (L - 1));
+    const int64_t u = t >> L_log2;
+    if (u >= n_chunks) return;
+    const int wl = threadIdx.x & 31;
+    const unsigned mask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << (wl & ~(L - 1)));
+    const int4 ch = chunks[u];
+    const int64_t v = ch.x;
+    const int o = lane >> w_log2;               // this lane's head
+    const bool active = o < op.H;
+    const int f0 = active ? o * op.D + (lane & (w - 1)) * VEC : 0;   // chunk j at f0 + j * w * VEC
+    const Operand &P = a_is_src ? op.A : op.B;  // gathered per edge (Src_V)
+    const Operand &Q = a_is_src ? op.B : op.A;  // hoisted (Dst_V, local row v)
+    const uint64_t keep = l2_policy_evict_last(), stream = l2_policy_evict_first();
+
+    float q[NJ][VEC];
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) {
+        if (active) ldg_vec<VEC>(Q.p + v * Q.ld + f0 + j * w * VEC, q[j]);
+        else
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) q[j][i] = 0.0f;
+    }
+    const float *__restrict__ Pb = P.p + f0;
+    const int jstride = w * VEC;
+    const int64_t ldp = P.ld;
+
+    float acc = g_init<GOP>();
+    auto edge_msg = [&](const float (&p)[NJ][VEC]) {
+        float s = 0.0f;
+#pragma unroll
+        for (int j = 0; j < NJ; ++j)
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) s = __fmaf_rn(p[j][i], q[j][i], s);
+        for (int off = w >> 1; off > 0; off >>= 1) s += __shfl_xor_sync(mask, s, off);
+        return s;
+    };
+    auto emit = [&](int k, float m) {
+        if constexpr (GOP == UG_GATHER_ASSIGN) {
+            if (active && (lane & (w - 1)) == 0) {
+                const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
+                op.C[e * op.c_ld + o] = m;
+            }
+        } else {
+            acc = g_combine<GOP>(acc, m);
+        }
+    };
+    int k = ch.y;                               // CSR positions are int32
+    const int k1 = ch.z;
+    for (; k + UE <= k1; k += UE) {
+        float p[UE][NJ][VEC];
+        int64_t s[UE];
+#pragma unroll
+        for (int e = 0; e < UE; ++e) s[e] = ldg_i32_hint(g.col + k + e, stream);
+#pragma unroll
+        for (int e = 0; e < UE; ++e) {
+#pragma unroll
+            for (int j = 0; j < NJ; ++j) {
+                if (active) ldg_vec_hint<VEC>(Pb + s[e] * ldp + j * jstride, p[e][j], keep);
+                else
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) p[e][j][i] = 0.0f;
+            }
+        }
+#pragma unroll
+        for (int e = 0; e < UE; ++e) emit(k + e, edge_msg(p[e]));
+    }
+    // one edge per step: the next edge's column index is loaded while this one is gathered
+    int64_t s_next = k < k1 ? ldg_i32_hint(g.col + k, stream) : 0;
+    for (; k < k1; ++k) {
+        float p[NJ][VEC];
+        const int64_t s = s_next;
+        if (k + 1 < k1) s_next = ldg_i32_hint(g.col + k + 1, stream);
+#pragma unroll
+        for (int j = 0; j < NJ; ++j) {
+            if (active) ldg_vec_hint<VEC>(Pb + s * ldp + j * jstride, p[j], keep);
+            else
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) p[j][i] = 0.0f;
+        }
+        emit(k, edge_msg(p));
+    }
+    if constexpr (GOP != UG_GATHER_ASSIGN) {
+        if (!active || (lane & (w - 1)) != 0) return;
+        if (ch.w < 0) {
+            const int64_t deg = (int64_t)k1 - ch.y;         // an owned row is one chunk: its whole in-edge list
+            op.C[v * op.c_ld + o] = g_finalize<GOP>(acc, deg);
+        } else {
+            scratch[(int64_t)ch.w * sld + o] = acc;
+        }
+    }
+}
+
+// NJ * VEC features per lane, one head per lane: D % (NJ * VEC) == 0 and w = D / (NJ * VEC)
+// a power of two; L = next power of two >= H * w, at most 32 -- the largest NJ that fits
+// (fewer butterfly steps per edge: measured on C4 F=128, 8 lanes x 16 features 98 us against
+// 32 lanes x 4 features 167 us).  Returns NJ, or 0 when the op does not fit (the caller then
+// uses the generic dot kernel).
+int dotsv_nj(const OpArgs &op, int vec, int *L, int *w) {
+    for (int nj : {4, 2, 1}) {
+        const int per = nj * vec;
+        if (op.D % per) continue;
+        const int ww = op.D / per;
+        if (ww & (ww - 1)) continue;
+        const int64_t lanes = (int64_t)op.H * ww;
+        if (lanes > 32) continue;
+        int l = 1;
+        while (l < lanes) l <<= 1;
+        *L = l;
+        *w = ww;
+        return nj;
+    }
+    return 0;
+}
+
+cudaError_t launch_dotsv(int gather, const GraphArgs &g, const OpArgs &op, bool a_is_src, int vec, int block,
+                         const SplitPlan &plan, float *scratch, cudaStream_t s, cudaEvent_t ev_begin,
+                         cudaEvent_t ev_end) {
+    int L = 0, w = 0;
+    const int nj = dotsv_nj(op, vec, &L, &w);
+    if (nj == 0) return cudaErrorInvalidValue;
+    const int64_t threads = plan.n_chunks * (int64_t)L;
+    if (threads == 0) return cudaSuccess;
+    const int64_t grid = cdiv(threads, block);
+    const int64_t sld = cdiv(op.W, 4) * 4;
+    const int4 *chunks = reinterpret_cast<const int4 *>(plan.d_chunk);
+    if (ev_begin) cudaEventRecord(ev_begin, s);
+#define UG_DOTSV(NJV)                                                                                     \
+    k_dotsv<GOP, VEC, NJV><<<(unsigned)grid, block, 0, s>>>(g, op, a_is_src, chunks, plan.n_chunks,      \
+                                                           ilog2(L), ilog2(w), scratch, sld)
+    UG_DISPATCH_VEC(vec, VEC,
+        UG_DISPATCH_GOP(gather, GOP, {
+            switch (nj) {
+            case 1: UG_DOTSV(1); break;
+            case 2: UG_DOTSV(2); break;
+            default: UG_DOTSV(4); break;
+            }
+        }));
+#undef UG_DOTSV
+    if (ev_end) cudaEventRecord(ev_end, s);
+    cudaError_t err = cudaGetLastError();
+    if (err != cudaSuccess || gather == UG_GATHER_ASSIGN || plan.n_split_rows == 0) return err;
+    const int64_t fgrid = cdiv(plan.n_split_rows * (int64_t)op.W, 256);
+    const int4 *split = reinterpret_cast<const int4 *>(plan.d_split);
+    UG_DISPATCH_RED(gather, GOP,
+        k_split_fix<GOP, 1><<<(unsigned)fgrid, 256, 0, s>>>(g, op, split, plan.n_split_rows, scratch, sld));
+    return cudaGetLastError();
+}
+
+}  // namespace ug

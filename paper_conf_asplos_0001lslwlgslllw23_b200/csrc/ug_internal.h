@@ -79,6 +79,11 @@ cudaError_t launch_split_vertex(int kedge, int gather, const GraphArgs &g, const
                                 cudaStream_t s, cudaEvent_t ev_begin = nullptr, cudaEvent_t ev_end = nullptr);
 cudaError_t launch_dot(bool vertex_units, int gather, const GraphArgs &g, const OpArgs &op,
                        const LaunchCfg &c, cudaStream_t s);
+// dot between a Src_V and a Dst_V operand under SV (k_dotsv.cu): Dst_V row hoisted per unit.
+int dotsv_nj(const OpArgs &op, int vec, int *L, int *w);
+cudaError_t launch_dotsv(int gather, const GraphArgs &g, const OpArgs &op, bool a_is_src, int vec, int block,
+                         const SplitPlan &plan, float *scratch, cudaStream_t s, cudaEvent_t ev_begin,
+                         cudaEvent_t ev_end);
 cudaError_t launch_init(int gather, const OpArgs &op, int64_t rows, cudaStream_t s);
 cudaError_t launch_epilogue(int gather, const GraphArgs &g, const OpArgs &op, cudaStream_t s);
 // Fused GAT attention chain (ug_gat_attention, k_gat.cu).

@@ -128,6 +128,21 @@ ug_status lower(const ug_graph *g, const ug_op_info *op, Lowered *out) {
 
 // ------------------------------------------------------------------------- resolution
 
+// dot under SV with one Src_V and one Dst_V full-width operand (u_dot_v / v_dot_u): k_dotsv,
+// which keeps the Dst_V row in registers per work unit.  Other dot ops under SV use k_dot.
+static bool dotsv_ok(const Lowered &lw, const LaunchCfg &c, bool *a_is_src = nullptr, int *L = nullptr) {
+    if (!lw.dot || c.strategy != UG_SV) return false;
+    const Operand &A = lw.args.A, &B = lw.args.B;
+    if (A.div != 1 || B.div != 1) return false;
+    const bool as = A.type == UG_T_SRC_V && B.type == UG_T_DST_V;
+    const bool bs = A.type == UG_T_DST_V && B.type == UG_T_SRC_V;
+    int l = 0, w = 0;
+    if ((!as && !bs) || dotsv_nj(lw.args, c.vec, &l, &w) == 0) return false;
+    if (a_is_src) *a_is_src = as;
+    if (L) *L = l;
+    return true;
+}
+
 ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, LaunchCfg *cfg) {
     (void)g;
     LaunchCfg c{};
@@ -170,7 +185,11 @@ ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, La
         c.L = L;
     }
     if (c.strategy == UG_BE) c.L = std::min(32, need);
-    if (c.strategy == UG_SV && lw.dot) c.G = 1;   // dot under SV: one row per lane group (k_dot)
+    if (c.strategy == UG_SV && lw.dot) {
+        int L = 0;
+        if (dotsv_ok(lw, c, nullptr, &L)) c.L = L;   // k_dotsv: SV chunks of G in-edges
+        else c.G = 1;                                 // other dot ops: one row per lane group (k_dot)
+    }
     *cfg = c;
     return UG_OK;
 }
@@ -256,7 +275,7 @@ static int launches_for(const Lowered &lw, const LaunchCfg &c, int64_t n_split_r
     const bool edge_units = c.strategy == UG_TE || c.strategy == UG_WE || c.strategy == UG_BE;
     if (lw.to_edges) return 1;
     if (edge_units) return lw.gather == UG_GATHER_SUM ? 2 : 3;
-    if (c.strategy == UG_SV && !lw.dot) return n_split_rows > 0 ? 2 : 1;
+    if (c.strategy == UG_SV && (!lw.dot || dotsv_ok(lw, c))) return n_split_rows > 0 ? 2 : 1;
     return 1;
 }
 
@@ -299,7 +318,7 @@ extern "C" ug_status ug_op_launch_count(const ug_graph *g, const ug_op_info *op,
     ug_status st = prepare(g, op, sched, &lw, &c);
     if (st != UG_OK) return st;
     int64_t nsr = 0;
-    if (c.strategy == UG_SV && !lw.dot && !lw.to_edges) {
+    if (c.strategy == UG_SV && (!lw.dot || dotsv_ok(lw, c)) && !lw.to_edges) {
         // count split rows on the host without touching the device
         for (int64_t v = 0; v < g->V; ++v)
             if ((int64_t)g->h_row_ptr[v + 1] - g->h_row_ptr[v] > c.G) ++nsr;
@@ -331,6 +350,18 @@ static ug_status run(const ug_graph *g, const ug_op_info *op, const ug_schedule 
             if (ev_end) cudaEventRecord(ev_end, s);
         }
         if (err == cudaSuccess && lw.gather != UG_GATHER_SUM) err = launch_epilogue(lw.gather, ga, lw.args, s);
+    } else if (bool a_src = false; dotsv_ok(lw, c, &a_src)) {
+        const SplitPlan *plan = nullptr;
+        if ((st = get_plan(g, c.G, &plan)) != UG_OK) return st;
+        float *scratch = nullptr;
+        const int64_t sld = (lw.args.W + 3) / 4 * 4;
+        if (agg && plan->n_split_chunks > 0) {
+            ensure_pool_retains();
+            err = cudaMallocAsync((void **)&scratch, sizeof(float) * (size_t)(plan->n_split_chunks * sld), s);
+            if (err != cudaSuccess) return set_error(UG_ERR_OOM, "SV scratch allocation failed");
+        }
+        err = launch_dotsv(lw.gather, ga, lw.args, a_src, c.vec, c.block, *plan, scratch, s, ev_begin, ev_end);
+        if (scratch) cudaFreeAsync(scratch, s);
     } else if (lw.dot) {
         if (ev_begin) cudaEventRecord(ev_begin, s);
         err = launch_dot(!edge_units, lw.gather, ga, lw.args, c, s);

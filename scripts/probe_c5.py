@@ -28,6 +28,7 @@ def main():
     ap.add_argument("--schedule", default="SV_G512_F128_P1")
     ap.add_argument("--reps", type=int, default=8)
     ap.add_argument("--F", type=int, default=602)
+    ap.add_argument("--modes", default="b2b,gap,flush,aligned")
     a = ap.parse_args()
     c = ugdata.CONFIGS[a.config]
     src, dst = ugdata.graph(a.config)
@@ -65,11 +66,17 @@ def main():
         print(f"{mode:8s} {sched:18s} step median {statistics.median(step):8.3f} ms  kernel median "
               f"{statistics.median(kern):8.3f} ms  min {min(kern):8.3f}", flush=True)
 
+    modes = a.modes.split(",")
+    from bench import ClockSampler
     for mode in ("b2b", "gap", "flush"):
-        run(mode, a.schedule, X, Y)
-    base = a.schedule.replace("_P1", "")
-    for mode in ("b2b", "gap"):
-        run(mode, base, Xa, Ya)
+        if mode in modes:
+            with ClockSampler(torch.cuda.current_device()) as cs:
+                run(mode, a.schedule, X, Y)
+            print("   clocks", cs.summary(), flush=True)
+    if "aligned" in modes:
+        base = a.schedule.replace("_P1", "")
+        for mode in ("b2b", "gap"):
+            run(mode, base, Xa, Ya)
 
 
 if __name__ == "__main__":

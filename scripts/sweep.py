@@ -64,14 +64,14 @@ def candidates(cls, F, E, quick=False):
             c += [f"SV_G{g}_F{f}" for g in (16, 32, 64, 128, 512, 2048) for f in fts]
             c += [f"SV_G{g}_F{f}_P1" for g in (32, 128, 512) for f in (64, 128) if f <= max(16, 2 * F)]
         else:
-            c += [f"SV_G{g}" for g in (256, 1024)]
+            c += [f"SV_G{g}" for g in (16, 32, 64, 128, 512, 1024)]
     else:
         c += [f"TE_G{g}_T{t}" for g in (1, 2, 4, 8) for t in Ts]
         c += [f"WE_G{g}_T1" for g in (1, 4, 16)]
         c += [f"TV_G1_T{t}" for t in Ts if t >= 4]
         c += [f"WV_G{g}_T1" for g in (1, 4)]
         c += ["BV_G1_B256", "BE_G256"]
-        c += [f"SV_G{g}" for g in (64, 512)]
+        c += [f"SV_G{g}" for g in ((16, 32, 64, 128, 512) if cls == "dot_msg" else (64, 512))]
     if E > 50_000_000:   # C5: drop the schedules that take seconds (atomic per-element TE at F=602)
         c = [s for s in c if not (s.startswith("TE") and cls.startswith("agg") and "_F" not in s) and not s.startswith("TV")
              and not s.startswith("WV")]
