@@ -38,7 +38,7 @@ def main():
     for V, src, dst in graphs():
         E = len(src)
         g = ug.Graph(V, src, dst)
-        for F, H in ((18, 3), (20, 1)):
+        for F, H in ((18, 3), (20, 1), (16, 1), (24, 3)):   # the last two also take k_dotsv
             X = torch.randn(V, F, device="cuda")
             w = torch.randn(E, H, device="cuda").abs() + 0.5
             for (eo, a, b, go, c) in OPS:
