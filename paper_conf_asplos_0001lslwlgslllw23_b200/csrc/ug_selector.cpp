@@ -5,7 +5,8 @@
 //  1. a table of schedules MEASURED on B200 for the named configs (scripts/sweep.py writes
 //     selector_table.json), keyed by the Table 7 features plus the feature width F that Fig. 7
 //     shows matters: op class, F, mean in-degree, degree CV (= std_nnz /
-//     mean), V -- first matching entry wins;
+//     mean), V -- among the entries whose ranges hold the graph, the nearest (log distance
+//     to the range centres) wins;
 //  2. a learned model (selector_model.txt, scripts/train_selector.py): per op class a
 //     cost-sensitive regression tree trained on a synthetic B200 corpus of graphs
 //     (scripts/selector_corpus.py), features log2 V, log2 E, log2 mean degree, CV,
@@ -266,12 +267,26 @@ ug_status select_schedule(const ug_graph *g, const Lowered &lw, ug_schedule *out
     const int classes[2] = {lw.op_class, (lw.op_class == 4 || lw.op_class == 5) ? 1 : -2};
     for (int pass = 0; pass < 2; ++pass) {
         if (classes[pass] == -2) break;
+        // among the entries whose box holds the graph, the nearest one wins: distance = sum over
+        // (F, mean degree, CV, V) of |log(x / geometric centre of the entry's range)| (boxes of
+        // neighbouring configs overlap, e.g. C3 and C4 share F = 128 and mean degree ~7-8)
+        const Entry *best = nullptr;
+        double best_d = 0;
+        auto ld = [](double x, double lo, double hi) {
+            if (lo <= 0 || hi >= 1e17) return 0.0;     // open range: no preference
+            return std::fabs(std::log(std::max(x, 1e-12) / std::sqrt(lo * hi)));
+        };
         for (const Entry &e : g_table) {
             if (e.op_class != -1 && e.op_class != classes[pass]) continue;
             if (F < e.F_lo || F > e.F_hi || deg < e.deg_lo || deg > e.deg_hi || cv < e.cv_lo || cv > e.cv_hi ||
                 V < e.V_lo || V > e.V_hi)
                 continue;
-            *out = adapt(lw, e.sched);
+            const double d = ld(F, e.F_lo, e.F_hi) + ld(deg, e.deg_lo, e.deg_hi) + ld(cv, e.cv_lo, e.cv_hi) +
+                             ld(V, e.V_lo, e.V_hi);
+            if (!best || d < best_d) { best = &e; best_d = d; }
+        }
+        if (best) {
+            *out = adapt(lw, best->sched);
             return UG_OK;
         }
         if (pass == 0) {
