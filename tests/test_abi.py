@@ -248,3 +248,30 @@ def test_selector_table_load_and_match(tmp_path):
         empty = tmp_path / "empty.json"
         empty.write_text('{"entries": []}')
         ug.selector_load(empty)
+
+
+def test_selector_table_nearest_entry_wins(tmp_path):
+    """Overlapping entries (neighbouring configs share F and degree ranges): the entry whose
+    range centres are nearest (log distance) to the graph's features wins, whatever the order."""
+    src, dst = ugdata.graph("C1")
+    V = ugdata.CONFIGS["C1"].V
+    g = host_graph(V, src, dst)
+    st = g.stats()
+    deg = st["mean_deg"]
+    X, Y = torch.zeros(V, 16), torch.zeros(V, 16)
+    far = (f'{{"class": "agg", "F_lo": 8, "F_hi": 20, "deg_lo": {deg / 3}, "deg_hi": {deg * 12}, '
+           f'"V_lo": 100, "V_hi": 1000000, "schedule": "WV_G1_T1"}}')
+    near = (f'{{"class": "agg", "F_lo": 8, "F_hi": 32, "deg_lo": {deg / 2}, "deg_hi": {deg * 2}, '
+            f'"V_lo": {V / 2}, "V_hi": {V * 2}, "schedule": "TE_G4_T4"}}')
+    ug.selector_load_model("")
+    try:
+        for entries in ([far, near], [near, far]):
+            t = tmp_path / "t.json"
+            t.write_text('{"version": 1, "entries": [' + ",".join(entries) + "]}")
+            ug.selector_load(t)
+            assert ug.schedule_select(g, "copy_lhs", "sum", A=X, a_type="u", C=Y, c_type="v") == "TE_G4_T4"
+    finally:
+        pkg = os.path.join(ROOT, "paper_conf_asplos_0001lslwlgslllw23_b200")
+        if os.path.exists(os.path.join(pkg, "selector_model.txt")):
+            ug.selector_load_model(os.path.join(pkg, "selector_model.txt"))
+        ug.selector_load(os.path.join(pkg, "selector_table.json"))
