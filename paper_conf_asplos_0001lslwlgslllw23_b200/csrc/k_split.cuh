@@ -89,6 +89,67 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
     for (; k < k1; k += UH) group(std::true_type{}, std::integral_constant<int, UH>{});
 }
 
+// Message creation (gather ASSIGN, C = Edge) on the fast path: the unit's in-edges are the
+// CSR positions [k, k1) (= edge ids), so each edge's message row is stored contiguously across
+// the unit's lanes; the Src_V row is gathered per edge, a Dst_V B operand is loaded once per
+// unit (BM 1), Edge / Src_V B operands per edge.  UF edges per step (loads first, then stores).
+template <int KE, int VEC, int BM>
+__device__ __forceinline__ void split_fast_assign(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t k,
+                                                  const int64_t k1, int f, int64_t cb) {
+    constexpr int UF = 2;
+    const float *__restrict__ Ab = op.A.p;
+    const uint64_t keep = l2_policy_evict_last(), stream = l2_policy_evict_first();
+    const uint32_t lda = (uint32_t)op.A.ld, fo = (uint32_t)f;
+    const uint32_t ldb = (uint32_t)op.B.ld, cbo = (uint32_t)cb;
+    constexpr bool bfull = BM == 3 || BM == 5;
+    const int nout = op.W - f;
+    const bool full_vec = nout >= VEC && op.c_vec >= VEC;
+    float bconst[VEC];
+    if constexpr (BM == 1) fetch<VEC>(op.B, v, cb, bconst);
+    auto one = [&](int64_t kk, uint32_t sq, float (&m)[VEC]) {
+        ldg_vec_hint<VEC>(Ab + (sq * lda + fo), m, keep);
+        if constexpr (BM != 0) {
+            float b[VEC];
+            if constexpr (BM == 1) {
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) b[i] = bconst[i];
+            } else {
+                const uint32_t row = (BM == 2 || BM == 3) ? (uint32_t)kk : sq;
+                const float *bp = op.B.p + (row * ldb + cbo);
+                if constexpr (bfull) {
+                    ldg_vec_hint<VEC>(bp, b, BM == 3 ? stream : keep);
+                } else {
+                    const float x = __ldg(bp);
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) b[i] = x;
+                }
+            }
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) m[i] = edge_fn<KE>(m[i], b[i]);
+        }
+    };
+    auto store = [&](int64_t kk, const float (&m)[VEC]) {
+        float *cp = op.C + kk * op.c_ld + f;
+        if (full_vec) st_vec_hint<VEC>(cp, m, stream);
+        else st_out<VEC>(cp, m, nout, op.c_vec);
+    };
+    for (; k + UF <= k1; k += UF) {
+        uint32_t sq[UF];
+#pragma unroll
+        for (int q = 0; q < UF; ++q) sq[q] = (uint32_t)ldg_i32_hint(g.col + k + q, stream);
+        float m[UF][VEC];
+#pragma unroll
+        for (int q = 0; q < UF; ++q) one(k + q, sq[q], m[q]);
+#pragma unroll
+        for (int q = 0; q < UF; ++q) store(k + q, m[q]);
+    }
+    for (; k < k1; ++k) {
+        float m[VEC];
+        one(k, (uint32_t)ldg_i32_hint(g.col + k, stream), m);
+        store(k, m);
+    }
+}
+
 #ifndef UG_BM2_MINB
 #define UG_BM2_MINB 5
 #endif
@@ -109,7 +170,9 @@ __device__ __forceinline__ void split_unit(const GraphArgs &g, const OpArgs &op,
     const int64_t ca = op_col(op.A, f);
     const int64_t cb = op_col(op.B, f);
 
-    if constexpr (GOP == UG_GATHER_ASSIGN) {
+    if constexpr (GOP == UG_GATHER_ASSIGN && FAST) {
+        split_fast_assign<KE, VEC, BM>(g, op, v, ch.y, k1, f, cb);
+    } else if constexpr (GOP == UG_GATHER_ASSIGN) {
         for (int64_t k = ch.y; k < k1; ++k) {
             const int64_t src = g.col[k];
             const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
@@ -232,7 +295,7 @@ cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, co
     // addressable with 32-bit element offsets (rows * ld < 2^32)
     const uint64_t lim = 1ull << 32;
     bool fast = op.A.type == UG_T_SRC_V && op.A.div == 1 && g.eid == nullptr &&
-                (uint64_t)g.V_src * (uint64_t)op.A.ld < lim && gather != UG_GATHER_ASSIGN;
+                (uint64_t)g.V_src * (uint64_t)op.A.ld < lim;
     if (KE != K_COPY) {
         const uint64_t brows = op.B.type == UG_T_EDGE ? (uint64_t)g.E : (uint64_t)g.V_src;
         fast = fast && brows * (uint64_t)op.B.ld < lim;
@@ -245,9 +308,7 @@ cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, co
                                                                  c.ftile, n_tiles, scratch, sld)
     UG_DISPATCH_VEC(c.vec, VEC,
         UG_DISPATCH_GOP(gather, GOP, {
-            if constexpr (GOP == UG_GATHER_ASSIGN) {
-                UG_SV_LAUNCH(-1);
-            } else if constexpr (KE == K_COPY) {
+            if constexpr (KE == K_COPY) {
                 if (bm == 0) UG_SV_LAUNCH(0); else UG_SV_LAUNCH(-1);
             } else {
                 switch (bm) {

@@ -71,7 +71,10 @@ def candidates(cls, F, E, quick=False):
         c += [f"TV_G1_T{t}" for t in Ts if t >= 4]
         c += [f"WV_G{g}_T1" for g in (1, 4)]
         c += ["BV_G1_B256", "BE_G256"]
-        c += [f"SV_G{g}" for g in ((16, 32, 64, 128, 512) if cls == "dot_msg" else (64, 512))]
+        if cls == "dot_msg":
+            c += [f"SV_G{g}" for g in (16, 32, 64, 128, 512)]
+        else:   # message creation under SV: row chunks x column tiles, Dst_V operand hoisted
+            c += [f"SV_G{g}_F{f}" for g in (16, 32, 64) for f in (16, 32, 64) if f <= max(16, F)]
     if E > 50_000_000:   # C5: drop the schedules that take seconds (atomic per-element TE at F=602)
         c = [s for s in c if not (s.startswith("TE") and cls.startswith("agg") and "_F" not in s) and not s.startswith("TV")
              and not s.startswith("WV")]
