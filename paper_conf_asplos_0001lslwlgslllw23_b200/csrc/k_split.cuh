@@ -97,7 +97,7 @@ template <int KE, int VEC, int BM>
 __device__ __forceinline__ void split_fast_assign(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t k,
                                                   const int64_t k1, int f, int64_t cb) {
 #ifndef UG_ASSIGN_UF
-#define UG_ASSIGN_UF 2
+#define UG_ASSIGN_UF 4
 #endif
     constexpr int UF = UG_ASSIGN_UF;
     const float *__restrict__ Ab = op.A.p;
@@ -242,7 +242,7 @@ __device__ __forceinline__ int unit_tile(int64_t u, int64_t n_chunks, int n_tile
 
 template <int KE, int GOP, int VEC, int BM>
 #ifndef UG_ASSIGN_MINB
-#define UG_ASSIGN_MINB 0
+#define UG_ASSIGN_MINB 6
 #endif
 __global__ void __launch_bounds__(256, (UG_ASSIGN_MINB > 0 && GOP == UG_GATHER_ASSIGN) ? UG_ASSIGN_MINB : (BM == 0) ? UG_BM0_MINB : (BM == 2 ? UG_BM2_MINB : (BM > 0 ? (VEC == 4 ? 5 : 6) : 4))) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
                                                int64_t n_chunks, int L_log2, int ftile, int n_tiles,
