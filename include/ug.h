@@ -90,8 +90,12 @@ typedef enum {
     UG_WE = 4,      /* warp-edge:     T warps per edge                                          */
     UG_BV = 5,      /* block-vertex:  one CTA per G rows, its warps split each row's edges     */
     UG_BE = 6,      /* block-edge:    one CTA per G x warps edges, contiguous, segmented reduce */
-    UG_SV = 7       /* split-vertex (B200): rows cut into <= `group` edge chunks, column tiles of
-                       `ftile` features in tile-major order (L2-resident), partials fixed up   */
+    UG_SV = 7       /* split-vertex (B200): rows cut into <= `group` edge chunks (scheduled
+                       longest first), column tiles of `ftile` features in tile-major order
+                       (L2-resident), partials of split rows fixed up in chunk order.  For
+                       `dot` between one Src_V and one Dst_V operand the Dst_V row is held in
+                       registers per chunk (ftile unused); message creation stores each edge's
+                       row contiguously (dst-sorted graphs)                                     */
 } ug_strategy;
 
 typedef struct {
