@@ -91,10 +91,10 @@ class Graph:
     def handle(self):
         return self._h
 
-    def __del__(self):
+    def __del__(self, _destroy=lib.ug_graph_destroy):   # bound at import: safe at interpreter exit
         h = getattr(self, "_h", None)
         if h is not None and h.value:
-            lib.ug_graph_destroy(h)
+            _destroy(h)
             self._h = None
 
     def stats(self):
