@@ -153,8 +153,14 @@ __device__ __forceinline__ void split_fast_assign(const GraphArgs &g, const OpAr
     }
 }
 
+// BM = 2 (per-edge scalar B, e.g. u_mul_e_sum): 6 CTAs / SM (40 registers, spill-free) for sum /
+// mean, measured 305 -> 291 us on C3 F = 128 and 82 -> 76 us at F = 32 (scripts/gpu_bm2.sh);
+// max / min and div keep 5 (48 registers: at 40 they spill 30-80 bytes per thread)
 #ifndef UG_BM2_MINB
 #define UG_BM2_MINB 5
+#endif
+#ifndef UG_BM2_SUM_MINB
+#define UG_BM2_SUM_MINB 6
 #endif
 #ifndef UG_BM0_MINB
 #define UG_BM0_MINB 8
@@ -244,7 +250,7 @@ template <int KE, int GOP, int VEC, int BM>
 #ifndef UG_ASSIGN_MINB
 #define UG_ASSIGN_MINB 6
 #endif
-__global__ void __launch_bounds__(256, (UG_ASSIGN_MINB > 0 && GOP == UG_GATHER_ASSIGN) ? UG_ASSIGN_MINB : (BM == 0) ? UG_BM0_MINB : (BM == 2 ? UG_BM2_MINB : (BM > 0 ? (VEC == 4 ? 5 : 6) : 4))) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
+__global__ void __launch_bounds__(256, (UG_ASSIGN_MINB > 0 && GOP == UG_GATHER_ASSIGN) ? UG_ASSIGN_MINB : (BM == 0) ? UG_BM0_MINB : (BM == 2 ? ((GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN) && KE != K_DIV ? UG_BM2_SUM_MINB : UG_BM2_MINB) : (BM > 0 ? (VEC == 4 ? 5 : 6) : 4))) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
                                                int64_t n_chunks, int L_log2, int ftile, int n_tiles,
                                                float *__restrict__ scratch, int64_t sld) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
