@@ -437,8 +437,46 @@ def main():
     torch.cuda.synchronize()
     tot = sum(ev_s0[i].elapsed_time(ev_s1[i]) for i in range(args.steps))
     ktot = sum(ev_k0[i].elapsed_time(ev_k1[i]) for i in range(args.steps))
+    t_p = None
     if world > 1:
-        tot, ktot = max_over_ranks([tot, ktot])
+        # T_P with and without the all-gather.  The exchange-free step runs the same
+        # local op(s) on the X already gathered (same buffers, same schedule), K times, timed the
+        # same way (barrier + sync on both sides, max over ranks).
+        def local_only():
+            if chunked:
+                for c, (c0, c1) in enumerate(bufs["cols"]):
+                    ug.op_run(g, eo, go, A=bufs["full"][c][:V], a_type="u", C=Y[:, c0:c1], c_type="v",
+                              F=c1 - c0, H=1)
+            else:
+                ug.op_run(g, eo, go, schedule=chosen, **kw)
+        local_only()
+        torch.cuda.synchronize()
+        dist.barrier()
+        torch.cuda.synchronize()
+        n0 = torch.cuda.Event(enable_timing=True)
+        n1 = torch.cuda.Event(enable_timing=True)
+        n0.record(stream)
+        for _ in range(args.steps):
+            local_only()
+        n1.record(stream)
+        torch.cuda.synchronize()
+        dist.barrier()
+        torch.cuda.synchronize()
+        g0 = torch.cuda.Event(enable_timing=True)
+        g1 = torch.cuda.Event(enable_timing=True)
+        g0.record(stream)
+        for _ in range(args.steps):
+            sh.gather_x(X_local, X_full)
+        g1.record(stream)
+        torch.cuda.synchronize()
+        tot, ktot, ntot, gtot = max_over_ranks([tot, ktot, n0.elapsed_time(n1), g0.elapsed_time(g1)])
+        t_p = {"with_allgather_ms": round(tot / args.steps, 4),
+              "without_allgather_ms": round(ntot / args.steps, 4),
+              "allgather_alone_ms": round(gtot / args.steps, 4),
+              "allgather_bytes_per_rank": int(sh.blk * (world - 1) * F * 4),
+              "how": "max over ranks of K steps, CUDA events on the launching stream; 'with' is the "
+                     "timed step (exchange overlapped by column chunks when chunked), 'without' the "
+                     "same local op(s) on the already-gathered X, 'alone' the unchunked all-gather"}
     ms = tot / args.steps
     kms = ktot / args.steps
     by = logical_bytes(V, E, F, args.op)
@@ -535,6 +573,7 @@ def main():
                             else " + NCCL all-gather of X") if world > 1 else ""),
                        "logical_bytes": by},
             "latency_ms": round(ms, 4),
+            **({"t_p": t_p} if t_p else {}),
             "graph_ingest_ms": round(ingest_ms, 1),
             "frac_of_8TBps": round(value / 8000.0, 4),
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
