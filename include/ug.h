@@ -107,12 +107,23 @@ typedef struct {
     int32_t block_threads;  /* CTA size (0 -> 256)                                              */
     int32_t ftile;          /* column-tile width for L2 blocking, tile-major grid order; 0 = off */
     int32_t vec;            /* feature vector width 1/2/4; 0 -> widest the layout allows        */
-    int32_t flags;          /* UG_SCHED_PACK (SV only): first stage a full-width Src_V operand whose
+    int32_t flags;          /* UG_SCHED_PACK | UG_SCHED_TMA | UG_SCHED_ASYNC.  UG_SCHED_PACK (SV only): first stage a full-width Src_V operand whose
                                rows are not 128-byte aligned into an aligned scratch copy, so each
                                column slab occupies whole L2 lines and rows take 16-byte loads   */
 } ug_schedule;
 
 #define UG_SCHED_PACK 1
+#define UG_SCHED_TMA  2   /* SV aggregation only ("_M1"): source rows are gathered four at a time
+                             by TMA (cp.async.bulk.tensor tile::gather4, issued by one lane per
+                             warp) into a per-warp ring of shared-memory stages completed on
+                             mbarriers, instead of into registers                                */
+#define UG_SCHED_ASYNC 4  /* SV aggregation only ("_A1"): the same ring filled by cp.async
+                             (LDGSTS, each lane its own features of the group's four rows).
+                             Both staged forms: ftile = 32 * vec columns (128 / 64 / 32), a
+                             full-width Src_V A (rows not aligned for the copy width are packed
+                             first), identity edge ids, B absent, Dst_V, or a per-head / scalar
+                             Edge tensor; otherwise UG_ERR_UNSUPPORTED_SCHEDULE.  Measured
+                             against the register SV kernel in profiles/r2_staged_ab.md         */
 
 /* Optional allocator for graph-owned device arrays (e.g. torch's caching allocator).
  * NULL -> cudaMallocAsync / cudaFreeAsync on the given stream. */
@@ -147,7 +158,9 @@ ug_status ug_graph_create_csr(int64_t num_vertices, int64_t num_edges, const int
                               const int32_t *col_idx, const int32_t *eid, int on_device, int flags,
                               const ug_allocator *alloc, void *stream, ug_graph **out);
 
-/* Frees a graph or a view.  A parent must outlive its views. */
+/* Frees a graph or a view.  A parent must outlive its views.  Synchronises the device first
+ * (cudaDeviceSynchronize), so kernels still reading the graph on any stream finish before its
+ * memory is released. */
 ug_status ug_graph_destroy(ug_graph *g);
 
 /* Table 7 graph features: V (dst rows), E, mean in-degree,

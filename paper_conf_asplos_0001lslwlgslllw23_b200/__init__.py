@@ -71,6 +71,12 @@ class Graph:
     def __init__(self, num_vertices, src=None, dst=None, *, host_only=False, stream=None, _handle=None,
                  _parent=None):
         self._parent = _parent
+        self._dims_cache = None
+        self._host_only = bool(host_only) if _parent is None else _parent._host_only
+        self._device = None
+        if not self._host_only:
+            import torch
+            self._device = _parent._device if _parent is not None else torch.cuda.current_device()
         if _handle is not None:
             self._h = _handle
             return
@@ -98,7 +104,7 @@ class Graph:
         st = lib.ug_graph_create_csr(int(num_vertices), int(kb.shape[0]), rp, cp, ep, rdev, flags, None,
                                      None if host_only else _current_stream(stream), ctypes.byref(h))
         check(st, "ug_graph_create_csr")
-        return cls(num_vertices, _handle=h)
+        return cls(num_vertices, host_only=host_only, _handle=h)
 
     @property
     def handle(self):
@@ -117,6 +123,16 @@ class Graph:
                                  ctypes.byref(std), ctypes.byref(mx)), "ug_graph_stats")
         return {"V": V.value, "E": E.value, "mean_deg": mean.value, "std_nnz": std.value,
                 "max_deg": mx.value}
+
+    def dims(self):
+        """(rows of a Src_V operand, rows of a Dst_V operand / aggregation output, rows of an Edge
+        operand / message output): (V_total, V, E) -- for a view, V and E are its local rows and
+        edges while Src_V operands still span the parent's vertex-id space."""
+        if self._dims_cache is None:
+            st = self.stats()
+            vsrc = self._parent.dims()[0] if self._parent is not None else st["V"]
+            self._dims_cache = (vsrc, st["V"], st["E"])
+        return self._dims_cache
 
     @property
     def num_rows(self):
@@ -151,7 +167,11 @@ class Graph:
         return Graph(0, _handle=h, _parent=self)
 
 
-def _tensor(x, ttype, rows_hint=None):
+def _tensor(x, ttype, graph=None):
+    """ug_tensor for one operand.  The C ABI has no row count, so the rows each tensor type
+    implies (Src_V: V_total, Dst_V: V, Edge: E, Graph.dims) are checked here, with the device and
+    the row stride: a short, overlapping or off-device tensor would otherwise be read or written
+    out of bounds by the kernels."""
     if x is None:
         return UgTensor(None, TTYPES[None], 0, 0)
     import torch
@@ -161,12 +181,23 @@ def _tensor(x, ttype, rows_hint=None):
         raise TypeError("operands must be float32")
     if x.dim() == 1:
         x = x.view(-1, 1)
-    if x.dim() != 2 or x.stride(1) != 1:
+    if x.dim() != 2 or (x.shape[1] > 1 and x.stride(1) != 1):
         raise ValueError("operands must be 2-D with unit column stride")
-    return UgTensor(x.data_ptr(), TTYPES[ttype], x.shape[1], max(x.stride(0), x.shape[1]))
+    if x.shape[0] > 1 and x.stride(0) < x.shape[1]:
+        raise ValueError("operand rows overlap (row stride < width, e.g. an expand()ed tensor)")
+    if graph is not None:
+        if graph._device is not None and (not x.is_cuda or x.device.index != graph._device):
+            raise ValueError(f"operands must live on the graph's device cuda:{graph._device}")
+        if ttype in TTYPES and ttype is not None:
+            vsrc, v, e = graph.dims()
+            need = {"u": vsrc, "v": v, "e": e}[ttype]
+            if x.shape[0] < need:
+                raise ValueError(f"a {ttype!r} operand needs {need} rows, got {x.shape[0]}")
+    ld = x.stride(0) if x.shape[0] > 1 else x.shape[1]
+    return UgTensor(x.data_ptr(), TTYPES[ttype], x.shape[1], max(ld, x.shape[1]))
 
 
-def _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H):
+def _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H, graph=None):
     if F is None:
         ref = A if A is not None else B
         F = ref.shape[1] if ref.dim() == 2 else 1
@@ -174,8 +205,8 @@ def _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H):
             H = C.shape[1] if C.dim() == 2 else 1
     if H is None:
         H = 1
-    return UgOpInfo(EDGE_OPS[edge_op], GATHER_OPS[gather_op], _tensor(A, a_type), _tensor(B, b_type),
-                    _tensor(C, c_type), int(F), int(H))
+    return UgOpInfo(EDGE_OPS[edge_op], GATHER_OPS[gather_op], _tensor(A, a_type, graph), _tensor(B, b_type, graph),
+                    _tensor(C, c_type, graph), int(F), int(H))
 
 
 def parse_schedule(text):
@@ -215,7 +246,7 @@ def op_run(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, 
     (automatic) or Table 9 notation such as "TE_G1_T16" / "SV_G2048_F64".
     Asynchronous on `stream` (default: torch's current stream).
     """
-    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H, graph)
     check(lib.ug_op_run(graph.handle, ctypes.byref(info), _sched(schedule), _current_stream(stream)),
           "ug_op_run")
     return C
@@ -225,7 +256,7 @@ def op_run_events(graph, edge_op, gather_op, ev_begin, ev_end, A=None, a_type=No
                   C=None, c_type="v", F=None, H=None, schedule=None, stream=None):
     """op_run that also records torch.cuda.Event pair (ev_begin, ev_end) around the main kernel
     (measurement hook, ug_op_run_events).  The events must have been recorded once before."""
-    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H, graph)
     check(lib.ug_op_run_events(graph.handle, ctypes.byref(info), _sched(schedule), _current_stream(stream),
                                ctypes.c_void_p(ev_begin.cuda_event), ctypes.c_void_p(ev_end.cuda_event)),
           "ug_op_run_events")
@@ -238,7 +269,7 @@ class PreparedOp:
 
     def __init__(self, graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, C=None,
                  c_type="v", F=None, H=None, schedule=None):
-        self.info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+        self.info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H, graph)
         check(lib.ug_op_validate(graph.handle, ctypes.byref(self.info)), "ug_op_validate")
         if schedule is None:
             self.sched = UgSchedule()
@@ -267,13 +298,13 @@ def prepare(graph, edge_op, gather_op, **kw):
 
 def validate(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, C=None, c_type="v",
              F=None, H=None):
-    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H, graph)
     check(lib.ug_op_validate(graph.handle, ctypes.byref(info)), "ug_op_validate")
 
 
 def schedule_select(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, C=None,
                     c_type="v", F=None, H=None):
-    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H, graph)
     s = UgSchedule()
     check(lib.ug_schedule_select(graph.handle, ctypes.byref(info), ctypes.byref(s)), "ug_schedule_select")
     return format_schedule(s)
@@ -281,7 +312,7 @@ def schedule_select(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_ty
 
 def launch_count(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, C=None, c_type="v",
                  F=None, H=None, schedule=None):
-    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H)
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, c_type, F, H, graph)
     n = ctypes.c_int32()
     check(lib.ug_op_launch_count(graph.handle, ctypes.byref(info), _sched(schedule), ctypes.byref(n)),
           "ug_op_launch_count")
@@ -340,11 +371,13 @@ def op_run_arg(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=No
     op_run would and returns arg [V, F] int32 = the supplying edge id (first on ties, -1 for
     zero in-degree rows)."""
     import torch
-    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, "v", F, H)
+    info = _op_info(edge_op, gather_op, A, a_type, B, b_type, C, "v", F, H, graph)
     if arg is None:
         arg = torch.empty(C.shape[0], C.shape[1], dtype=torch.int32, device=C.device)
     if arg.dtype != torch.int32 or arg.dim() != 2 or arg.stride(1) != 1:
         raise TypeError("arg must be a 2-D int32 tensor with unit column stride")
+    if not arg.is_cuda or arg.device != C.device or arg.shape[0] < C.shape[0] or arg.shape[1] < C.shape[1]:
+        raise ValueError("arg must be an int32 CUDA tensor on C's device with at least C's shape")
     check(lib.ug_op_run_arg(graph.handle, ctypes.byref(info), arg.data_ptr(), max(arg.stride(0), arg.shape[1]),
                             _current_stream(stream)), "ug_op_run_arg")
     return arg
@@ -353,6 +386,15 @@ def op_run_arg(graph, edge_op, gather_op, A=None, a_type=None, B=None, b_type=No
 def arg_scatter(graph, arg, grad, target_type, out, stream=None):
     """out[row(e)][f / (W / out_width)] += grad[v][f] for e = arg[v][f] >= 0 (ug_arg_scatter);
     target_type "u" (row = src of e) or "e" (row = e)."""
+    import torch
+    if not isinstance(arg, torch.Tensor) or arg.dtype != torch.int32 or not arg.is_cuda or arg.dim() != 2 \
+            or arg.stride(1) != 1:
+        raise TypeError("arg must be a 2-D int32 CUDA tensor with unit column stride (from op_run_arg)")
+    if arg.shape[0] < graph.dims()[1] or grad.shape[0] < graph.dims()[1] or grad.shape[1] != arg.shape[1]:
+        raise ValueError("arg / grad need one row per destination vertex and equal widths")
+    rows_out = graph.dims()[0] if target_type == "u" else graph.dims()[2]
+    if out.shape[0] < rows_out:
+        raise ValueError(f"out needs {rows_out} rows")
     W = int(arg.shape[1])
     pg, lg = _mat(grad, "grad")
     po, lo = _mat(out, "out")
@@ -388,8 +430,11 @@ def rows_gather(X, idx, out=None, stream=None):
 
 
 class Renumbered:
-    """A graph renumbered for locality: `graph` is built on the new ids; to_new(X) / to_old(Y)
-    move vertex tensors between numberings on the device.  Edge ids are unchanged."""
+    """A graph renumbered for locality: `graph` is built on the new vertex ids from the COO
+    re-sorted by new destination, so its EDGE IDS ARE NEW TOO (the new CSR positions).
+    to_new(X) / to_old(Y) move vertex tensors between numberings; edges_to_new(W) moves an
+    edge tensor given in the original edge-id order into the new order (before a call), and
+    edges_to_old(M) moves an edge output (message creation, GAT attention) back (after)."""
 
     def __init__(self, num_vertices, src, dst, method="rcm"):
         import torch
@@ -406,6 +451,9 @@ class Renumbered:
         self._perm_d = torch.from_numpy(self.perm).cuda()
         self._inv_d = torch.from_numpy(self.inv).cuda()
         self._eord_d = torch.from_numpy(self.edge_order).cuda()
+        inv_e = np.empty_like(self.edge_order)
+        inv_e[self.edge_order] = np.arange(len(self.edge_order), dtype=np.int32)
+        self._einv_d = torch.from_numpy(inv_e).cuda()       # original edge id -> new position
 
     def to_new(self, X):
         return rows_gather(X, self._perm_d)
@@ -416,3 +464,7 @@ class Renumbered:
     def edges_to_new(self, W):
         """Edge tensor in original edge-id order -> the renumbered graph's edge order."""
         return rows_gather(W, self._eord_d)
+
+    def edges_to_old(self, M):
+        """Edge tensor in the renumbered graph's edge order -> original edge-id order."""
+        return rows_gather(M, self._einv_d)

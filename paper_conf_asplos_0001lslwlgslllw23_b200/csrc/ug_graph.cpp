@@ -194,11 +194,14 @@ extern "C" ug_status ug_graph_create_csr(int64_t V, int64_t E, const int32_t *ro
 extern "C" ug_status ug_graph_destroy(ug_graph *g) {
     if (!g) return UG_ERR_INVALID_ARG;
     if (!g->host_only) {
+        // kernels on any stream (torch's non-blocking streams included) may still read the CSR or
+        // the plans: wait for the device before the memory can be handed to another allocation
+        cudaDeviceSynchronize();
         for (void *p : g->owned) {
             if (g->has_alloc) g->alloc.free(p, g->alloc.ctx, nullptr);
-            else cudaFreeAsync(p, nullptr);
+            else cudaFree(p);
         }
-        for (void *p : g->plan_allocs) cudaFreeAsync(p, nullptr);
+        for (void *p : g->plan_allocs) cudaFree(p);
     }
     delete g;
     return UG_OK;

@@ -55,6 +55,9 @@ struct LaunchCfg {
     int ftile;        // column tile width (multiple of vec), 0 = whole width
     int vec;          // 1, 2, 4
     bool pack;        // UG_SCHED_PACK: stage A into 128-byte-aligned rows first (SV only)
+    bool dott;        // SV dot with column tiles (k_dott): any head width, tile-major partials
+    int staged;       // SV aggregation with shared-memory row staging (k_svg): 0 off,
+                      // 1 UG_SCHED_TMA (TMA gather4), 2 UG_SCHED_ASYNC (cp.async / LDGSTS)
 };
 
 // Split-row plan for UG_SV (built once per (graph, chunk size), cached on the graph).
@@ -77,6 +80,17 @@ cudaError_t launch_block_vertex(int kedge, int gather, const GraphArgs &g, const
 cudaError_t launch_split_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
                                 const LaunchCfg &c, const SplitPlan &plan, float *scratch,
                                 cudaStream_t s, cudaEvent_t ev_begin = nullptr, cudaEvent_t ev_end = nullptr);
+// SV with shared-memory row staging (k_svg.cu): mode 0 TMA gather4, 1 cp.async; bm = B addressing
+// mode (0 none, 1 Dst_V, 2 Edge broadcast).
+bool svg_supported(const OpArgs &op, int vec, int mode);
+cudaError_t launch_split_staged(int mode, int kedge, int gather, const GraphArgs &g, const OpArgs &op, int vec,
+                                int bm, const SplitPlan &plan, float *scratch, cudaStream_t s, cudaEvent_t ev_begin,
+                                cudaEvent_t ev_end);
+// dot between a Src_V and a Dst_V operand for any head width (k_dott.cu)
+int dott_tiles(const OpArgs &op, int vec);
+cudaError_t launch_dott(const GraphArgs &g, const OpArgs &op, bool a_is_src, int vec, const SplitPlan &plan,
+                        float *C, int64_t c_ld, float *part, cudaStream_t s, cudaEvent_t ev_begin,
+                        cudaEvent_t ev_end);
 cudaError_t launch_dot(bool vertex_units, int gather, const GraphArgs &g, const OpArgs &op,
                        const LaunchCfg &c, cudaStream_t s);
 // dot between a Src_V and a Dst_V operand under SV (k_dotsv.cu): Dst_V row hoisted per unit.
@@ -142,9 +156,6 @@ struct ug_graph {
     // UG_SV plans keyed by chunk size.
     mutable std::mutex mu;
     mutable std::map<int, ug::SplitPlan> plans;
-    // per-(split row, column tile) arrival counters of single-launch split-row merges
-    // (ug_gat_attention), keyed by chunk size * 65536 + column tiles; zero between calls
-    mutable std::map<int64_t, int32_t *> counters;
     // src vertex by edge id (device), built on first use when eid is not the identity
     mutable int32_t *d_src_of_eid = nullptr;
     mutable std::vector<void *> plan_allocs;

@@ -152,6 +152,60 @@ ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, La
     // SV stores through any C alignment (st_out), so its vector width is bounded by the operands
     // only; with UG_SCHED_PACK the staged copy of A is 16-byte aligned (a_vec = 4).
     c.pack = c.strategy == UG_SV && (s.flags & UG_SCHED_PACK) && lw.pack_ok;
+    c.staged = (s.flags & UG_SCHED_TMA) ? 1 : ((s.flags & UG_SCHED_ASYNC) ? 2 : 0);
+    if (c.staged) {
+        // shared-memory row staging (k_svg): SV aggregation only; a misaligned A is packed first
+        if (c.strategy != UG_SV || lw.dot || lw.to_edges)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "staged SV (_M1 / _A1): SV aggregation of an elementwise message only");
+        const Operand &A = lw.args.A;
+        if (A.type != UG_T_SRC_V || A.div != 1)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "staged SV (_M1 / _A1): A must be a full-width Src_V operand");
+        const int ft = s.ftile > 0 ? s.ftile : (lw.args.W >= 128 ? 128 : (lw.args.W >= 64 ? 64 : 32));
+        if (ft != 32 && ft != 64 && ft != 128)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "staged SV (_M1 / _A1): ftile must be 32, 64 or 128");
+        c.ftile = ft;
+        c.vec = ft / 32;
+        if (s.vec && s.vec != c.vec)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "staged SV (_M1 / _A1): vec is ftile / 32");
+        const int need = c.staged == 1 ? 4 : c.vec;     // TMA rows: 16-byte aligned; cp.async: the copy width
+        if ((uintptr_t)A.p % (4 * need) != 0 || A.ld % need != 0) {
+            if (!lw.pack_ok) return set_error(UG_ERR_ALIGNMENT, "staged SV: A rows are not aligned for the copy width");
+            c.pack = true;
+        }
+        c.G = s.group > 0 ? s.group : 2048;
+        c.L = 32;
+        c.block = 32 * 4;
+        *cfg = c;
+        return UG_OK;
+    }
+    if (c.strategy == UG_SV && lw.dot && s.ftile > 0) {
+        // k_dott: column tiles of 32 * vec features of each head, any D (ftile = the widest tile)
+        const Operand &A = lw.args.A, &B = lw.args.B;
+        const bool as = A.type == UG_T_SRC_V && B.type == UG_T_DST_V;
+        const bool bs = A.type == UG_T_DST_V && B.type == UG_T_SRC_V;
+        if (!(as || bs) || A.div != 1 || B.div != 1)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "SV dot with ftile: one full-width Src_V and one Dst_V operand");
+        if (s.ftile != 32 && s.ftile != 64 && s.ftile != 128)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "SV dot: ftile must be 32, 64 or 128");
+        const Operand &P = as ? A : B, &Q = as ? B : A;
+        auto fits = [&](const Operand &o, int v) { return (uintptr_t)o.p % (4 * v) == 0 && o.ld % v == 0; };
+        const bool same = P.p == Q.p && P.ld == Q.ld;          // u_dot_v of one matrix with itself
+        c.pack = false;
+        int v = s.ftile / 32;
+        // widest v <= ftile / 32 with D % v == 0 and Q's rows aligned for v (P is packed into
+        // 128-byte rows when its own rows are not; a Q that is the same matrix follows it)
+        for (; v > 1; v >>= 1)
+            if (lw.args.D % v == 0 && (fits(Q, v) || same)) break;
+        if (v > 1 && !fits(P, v)) c.pack = true;
+        if (s.vec && s.vec != v) return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "SV dot: vec follows ftile and the layout");
+        c.dott = true;
+        c.vec = v;
+        c.ftile = 32 * v;
+        c.G = s.group > 0 ? s.group : 256;
+        c.L = 32;
+        *cfg = c;
+        return UG_OK;
+    }
     const int sv_vec = std::min(c.pack ? 4 : lw.a_vec, lw.b_vec);
     const int allowed = (c.strategy == UG_SV && !lw.dot) ? sv_vec : lw.max_vec;
     c.vec = s.vec ? s.vec : allowed;
@@ -208,11 +262,21 @@ static GraphArgs graph_args(const ug_graph *g) {
     return a;
 }
 
-// Split-row plan for UG_SV (cached per chunk size; uploaded synchronously on first use).
+// Restores this thread's stream-capture mode on scope exit.
+struct RelaxedCapture {
+    cudaStreamCaptureMode prev = cudaStreamCaptureModeRelaxed;
+    RelaxedCapture() { cudaThreadExchangeStreamCaptureMode(&prev); }
+    ~RelaxedCapture() { cudaThreadExchangeStreamCaptureMode(&prev); }
+};
+
+// Split-row plan for UG_SV (cached per chunk size; uploaded synchronously on first use).  The
+// one-time upload (cudaMalloc + cudaMemcpy, not stream work) runs in relaxed capture mode, so
+// the first call on a graph may itself be inside a CUDA-graph capture.
 static ug_status get_plan(const ug_graph *g, int G, const SplitPlan **out) {
     std::lock_guard<std::mutex> lock(g->mu);
     auto it = g->plans.find(G);
     if (it != g->plans.end()) { *out = &it->second; return UG_OK; }
+    RelaxedCapture relaxed;
     std::vector<int32_t> chunks, split, slot_row;
     int64_t slot = 0;
     for (int64_t v = 0; v < g->V; ++v) {
@@ -272,6 +336,10 @@ static ug_status get_plan(const ug_graph *g, int G, const SplitPlan **out) {
 }
 
 static int launches_for(const Lowered &lw, const LaunchCfg &c, int64_t n_split_rows) {
+    if (c.dott) {
+        const int msg = 1 + (dott_tiles(lw.args, c.vec) > 1 ? 1 : 0);
+        return lw.to_edges ? msg : msg + (n_split_rows > 0 ? 2 : 1);
+    }
     const bool edge_units = c.strategy == UG_TE || c.strategy == UG_WE || c.strategy == UG_BE;
     if (lw.to_edges) return 1;
     if (edge_units) return lw.gather == UG_GATHER_SUM ? 2 : 3;
@@ -318,7 +386,7 @@ extern "C" ug_status ug_op_launch_count(const ug_graph *g, const ug_op_info *op,
     ug_status st = prepare(g, op, sched, &lw, &c);
     if (st != UG_OK) return st;
     int64_t nsr = 0;
-    if (c.strategy == UG_SV && (!lw.dot || dotsv_ok(lw, c)) && !lw.to_edges) {
+    if (c.strategy == UG_SV && (!lw.dot || dotsv_ok(lw, c) || c.dott) && !lw.to_edges) {
         // count split rows on the host without touching the device
         for (int64_t v = 0; v < g->V; ++v)
             if ((int64_t)g->h_row_ptr[v + 1] - g->h_row_ptr[v] > c.G) ++nsr;
@@ -350,6 +418,74 @@ static ug_status run(const ug_graph *g, const ug_op_info *op, const ug_schedule 
             if (ev_end) cudaEventRecord(ev_end, s);
         }
         if (err == cudaSuccess && lw.gather != UG_GATHER_SUM) err = launch_epilogue(lw.gather, ga, lw.args, s);
+    } else if (c.dott) {
+        // dot messages by column tiles (k_dott); an aggregation reduces them with SV afterwards
+        const SplitPlan *plan = nullptr;
+        if ((st = get_plan(g, c.G, &plan)) != UG_OK) return st;
+        OpArgs args = lw.args;
+        const bool a_src = args.A.type == UG_T_SRC_V;
+        Operand &P = a_src ? args.A : args.B;
+        Operand &Q = a_src ? args.B : args.A;
+        float *packed = nullptr, *part = nullptr, *msg = nullptr;
+        ensure_pool_retains();
+        auto release = [&]() {
+            if (part) cudaFreeAsync(part, s);
+            if (msg) cudaFreeAsync(msg, s);
+            if (packed) cudaFreeAsync(packed, s);
+        };
+        if (c.pack) {
+            const int64_t ldp = (int64_t)(lw.args.F + 31) / 32 * 32;
+            if (cudaMallocAsync((void **)&packed, sizeof(float) * (size_t)(g->V_total * ldp), s) != cudaSuccess)
+                return set_error(UG_ERR_OOM, "SV dot pack allocation failed");
+            if (cudaMemcpy2DAsync(packed, sizeof(float) * ldp, P.p, sizeof(float) * P.ld, sizeof(float) * lw.args.F,
+                                  (size_t)g->V_total, cudaMemcpyDeviceToDevice, s) != cudaSuccess) {
+                release();
+                return set_error(UG_ERR_CUDA, "SV dot pack copy failed");
+            }
+            if (Q.p == P.p && Q.ld == P.ld) { Q.p = packed; Q.ld = ldp; }
+            P.p = packed;
+            P.ld = ldp;
+        }
+        if ((uint64_t)g->V_total * (uint64_t)P.ld >= (1ull << 32)) {
+            release();
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "SV dot: Src_V operand above 2^32 elements");
+        }
+        const int th = dott_tiles(args, c.vec);
+        const int64_t EH = g->E * (int64_t)lw.args.H;
+        if (th > 1 && EH > 0 &&
+            cudaMallocAsync((void **)&part, sizeof(float) * (size_t)(th * EH), s) != cudaSuccess) {
+            release();
+            return set_error(UG_ERR_OOM, "SV dot partial allocation failed");
+        }
+        float *dst = lw.args.C;
+        int64_t dld = lw.args.c_ld;
+        if (agg) {
+            if (EH > 0 && cudaMallocAsync((void **)&msg, sizeof(float) * (size_t)EH, s) != cudaSuccess) {
+                release();
+                return set_error(UG_ERR_OOM, "SV dot message allocation failed");
+            }
+            dst = msg;
+            dld = lw.args.H;
+        }
+        err = launch_dott(ga, args, a_src, c.vec, *plan, dst, dld, part, s, ev_begin, ev_end);
+        if (err == cudaSuccess && agg) {
+            // reduce the messages into Dst_V: copy_e_<gather> over the same chunks
+            ug_op_info red{};
+            red.edge_op = UG_EDGE_COPY_LHS;
+            red.gather_op = lw.gather;
+            red.A = ug_tensor{msg, UG_T_EDGE, lw.args.H, lw.args.H};
+            red.B = ug_tensor{nullptr, UG_T_NULL, 0, 0};
+            red.C = ug_tensor{lw.args.C, UG_T_DST_V, lw.args.H, lw.args.c_ld};
+            red.feat = lw.args.H;
+            red.heads = lw.args.H;
+            ug_schedule rs{};
+            rs.strategy = UG_SV;
+            rs.group = c.G;
+            st = run(g, &red, &rs, stream, nullptr, nullptr);
+            release();
+            return st;
+        }
+        release();
     } else if (bool a_src = false; dotsv_ok(lw, c, &a_src)) {
         const SplitPlan *plan = nullptr;
         if ((st = get_plan(g, c.G, &plan)) != UG_OK) return st;
@@ -401,7 +537,26 @@ static ug_status run(const ug_graph *g, const ug_op_info *op, const ug_schedule 
             err = cudaMallocAsync((void **)&scratch, sizeof(float) * (size_t)(plan->n_split_chunks * sld), s);
             if (err != cudaSuccess) return set_error(UG_ERR_OOM, "SV scratch allocation failed");
         }
-        err = launch_split_vertex(lw.kedge, lw.gather, ga, args, c, *plan, scratch, s, ev_begin, ev_end);
+        if (c.staged) {
+            // B addressing mode of k_svg: none, Dst_V (any width), or a per-head / scalar Edge tensor
+            int bm = -1;
+            if (lw.kedge == K_COPY) bm = 0;
+            else if (args.B.type == UG_T_DST_V) bm = 1;
+            else if (args.B.type == UG_T_EDGE && args.B.div > 1 && (uint64_t)g->E * (uint64_t)args.B.ld < (1ull << 32)) bm = 2;
+            const int mode = c.staged - 1;
+            if (bm < 0 || g->d_eid != nullptr || (uint64_t)g->V_total * (uint64_t)args.A.ld >= (1ull << 32) ||
+                !svg_supported(args, c.vec, mode)) {
+                if (scratch) cudaFreeAsync(scratch, s);
+                if (packed) cudaFreeAsync(packed, s);
+                return set_error(UG_ERR_UNSUPPORTED_SCHEDULE,
+                                 "staged SV: needs identity edge ids, an aligned A below 2^32 elements and B absent, "
+                                 "Dst_V or a per-head Edge tensor");
+            }
+            err = launch_split_staged(mode, lw.kedge, lw.gather, ga, args, c.vec, bm, *plan, scratch, s, ev_begin,
+                                      ev_end);
+        } else {
+            err = launch_split_vertex(lw.kedge, lw.gather, ga, args, c, *plan, scratch, s, ev_begin, ev_end);
+        }
         if (scratch) cudaFreeAsync(scratch, s);
         if (packed) cudaFreeAsync(packed, s);
     }
@@ -454,6 +609,8 @@ extern "C" ug_status ug_schedule_parse(const char *text, ug_schedule *out) {
         case 'F': s.ftile = (int32_t)val; break;
         case 'V': s.vec = (int32_t)val; break;
         case 'P': s.flags = val ? (s.flags | UG_SCHED_PACK) : (s.flags & ~UG_SCHED_PACK); break;
+        case 'M': s.flags = val ? (s.flags | UG_SCHED_TMA) : (s.flags & ~UG_SCHED_TMA); break;
+        case 'A': s.flags = val ? (s.flags | UG_SCHED_ASYNC) : (s.flags & ~UG_SCHED_ASYNC); break;
         default: return set_error(UG_ERR_INVALID_ARG, "bad schedule token '" + tok + "'");
         }
         pos = nxt;
@@ -473,6 +630,8 @@ extern "C" ug_status ug_schedule_format(const ug_schedule *s, char *buf, size_t 
         if (s->block_threads) r += "_B" + std::to_string(s->block_threads);
         if (s->vec) r += "_V" + std::to_string(s->vec);
         if (s->flags & UG_SCHED_PACK) r += "_P1";
+        if (s->flags & UG_SCHED_TMA) r += "_M1";
+        if (s->flags & UG_SCHED_ASYNC) r += "_A1";
     }
     std::snprintf(buf, len, "%s", r.c_str());
     return UG_OK;
@@ -499,23 +658,6 @@ extern "C" const char *ug_version(void) { return "ugraph-b200 0.1 (sm_100a)"; }
 
 // ------------------------------------------------------------------------- fused GAT chain
 namespace ug {
-// Arrival counters for single-launch split-row merges: n_split_rows x n_tiles int32, zeroed
-// once (synchronously) at first use; every call leaves them zero again.
-static ug_status get_counters(const ug_graph *g, int G, int n_tiles, int64_t n_split_rows, int32_t **out) {
-    std::lock_guard<std::mutex> lock(g->mu);
-    const int64_t key = (int64_t)G * 65536 + n_tiles;
-    auto it = g->counters.find(key);
-    if (it != g->counters.end()) { *out = it->second; return UG_OK; }
-    void *d = nullptr;
-    const size_t bytes = std::max<size_t>(16, (size_t)n_split_rows * n_tiles * 4);
-    if (cudaMalloc(&d, bytes) != cudaSuccess) return set_error(UG_ERR_OOM, "counter allocation failed");
-    g->plan_allocs.push_back(d);
-    if (cudaMemset(d, 0, bytes) != cudaSuccess) return set_error(UG_ERR_CUDA, "counter init failed");
-    g->counters.emplace(key, (int32_t *)d);
-    *out = (int32_t *)d;
-    return UG_OK;
-}
-
 static bool aligned(const void *p, int64_t ld, int vec) {
     return ((uintptr_t)p % (4 * vec)) == 0 && ld % vec == 0;
 }
@@ -549,8 +691,6 @@ extern "C" ug_status ug_gat_attention(const ug_graph *g, const float *el, int64_
     if (st != UG_OK) return st;
     if (plan->n_chunks * n_tiles >= (int64_t)1 << 31)
         return set_error(UG_ERR_SHAPE, "ug_gat_attention: more than 2^31 (chunk, tile) units");
-    int32_t *counters = nullptr;
-    if ((st = get_counters(g, G, n_tiles, plan->n_split_rows, &counters)) != UG_OK) return st;
     GatArgs a;
     a.el = el; a.er = er; a.z = z;
     a.ld_el = ld_el; a.ld_er = ld_er; a.ld_z = ld_z;
@@ -558,12 +698,21 @@ extern "C" ug_status ug_gat_attention(const ug_graph *g, const float *el, int64_
     a.F = F; a.H = H; a.D = D; a.slope = slope;
     cudaStream_t s = (cudaStream_t)stream;
     const int64_t sld = (F + 3) / 4 * 4, nfc = (F + vec - 1) / vec;
+    // split-row partials, then the per-call arrival counters of the last-arriver merge (one per
+    // (split row, column tile), zeroed on this stream): calls on other streams never share them
     float *scratch = nullptr;
+    int32_t *counters = nullptr;
     if (plan->n_split_chunks > 0) {
         ensure_pool_retains();
-        const size_t bytes = sizeof(float) * (size_t)plan->n_split_chunks * (size_t)(sld + 2 * nfc);
-        if (cudaMallocAsync((void **)&scratch, bytes, s) != cudaSuccess)
+        const size_t part = sizeof(float) * (size_t)plan->n_split_chunks * (size_t)(sld + 2 * nfc);
+        const size_t cnt = sizeof(int32_t) * (size_t)plan->n_split_rows * (size_t)n_tiles;
+        if (cudaMallocAsync((void **)&scratch, part + cnt, s) != cudaSuccess)
             return set_error(UG_ERR_OOM, "ug_gat_attention: scratch allocation failed");
+        counters = reinterpret_cast<int32_t *>(reinterpret_cast<char *>(scratch) + part);
+        if (cudaMemsetAsync(counters, 0, cnt, s) != cudaSuccess) {
+            cudaFreeAsync(scratch, s);
+            return set_error(UG_ERR_CUDA, "ug_gat_attention: counter init failed");
+        }
     }
     float *sst = scratch ? scratch + plan->n_split_chunks * sld : nullptr;
     cudaError_t e = launch_gat(graph_args(g), a, vec, L, *plan, plan->d_slot_row, scratch, sst, sld, nfc,
@@ -595,15 +744,22 @@ extern "C" ug_status ug_op_run_arg(const ug_graph *g, const ug_op_info *op, int3
     if ((st = get_plan(g, G, &plan)) != UG_OK) return st;
     if (plan->n_chunks * n_tiles >= (int64_t)1 << 31)
         return set_error(UG_ERR_SHAPE, "ug_op_run_arg: more than 2^31 (chunk, tile) units");
-    int32_t *counters = nullptr;
-    if ((st = get_counters(g, G, n_tiles, plan->n_split_rows, &counters)) != UG_OK) return st;
     cudaStream_t s = (cudaStream_t)stream;
     const int64_t sld = (W + 3) / 4 * 4;
     float *scratch = nullptr;
+    int32_t *counters = nullptr;
     if (plan->n_split_chunks > 0) {
+        // partial values + partial args, then per-call arrival counters zeroed on this stream
         ensure_pool_retains();
-        if (cudaMallocAsync((void **)&scratch, (size_t)plan->n_split_chunks * sld * 8, s) != cudaSuccess)
+        const size_t part = (size_t)plan->n_split_chunks * sld * 8;
+        const size_t cnt = sizeof(int32_t) * (size_t)plan->n_split_rows * (size_t)n_tiles;
+        if (cudaMallocAsync((void **)&scratch, part + cnt, s) != cudaSuccess)
             return set_error(UG_ERR_OOM, "ug_op_run_arg: scratch allocation failed");
+        counters = reinterpret_cast<int32_t *>(reinterpret_cast<char *>(scratch) + part);
+        if (cudaMemsetAsync(counters, 0, cnt, s) != cudaSuccess) {
+            cudaFreeAsync(scratch, s);
+            return set_error(UG_ERR_CUDA, "ug_op_run_arg: counter init failed");
+        }
     }
     int32_t *sarg = scratch ? reinterpret_cast<int32_t *>(scratch + plan->n_split_chunks * sld) : nullptr;
     cudaError_t e = launch_argext(lw.kedge, lw.gather, graph_args(g), lw.args, L, *plan, plan->d_slot_row, scratch,

