@@ -177,6 +177,40 @@ def gat(V, src, dst, el, er, z, H, slope=0.2, bound=False):
     return (out, attn[:E], bnd) if bound else (out, attn[:E])
 
 
+def dot_attention(V, src, dst, q, k, val, H, scale=None, bound=False):
+    """Dot-product attention chain (FusedMM-style SDDMM + softmax + SpMM, PAPER.md:588
+    and :224) by definition, fp64: per head, s_e = scale * <q[dst], k[src]>, softmax over each
+    destination's in-edges, out = sum_e a_e val[src].  q: [V, H*Dk], k: [V, H*Dk], val: [V, H*Dv]
+    float32; scale defaults to 1/sqrt(Dk).  Returns (out [V, H*Dv], attn [E, H]) float64, plus the
+    tolerance scale sum_e a_e |val| when bound=True."""
+    lib = _load()
+    if not hasattr(lib, "_dotattn_ready"):
+        p, i64, ci = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int
+        lib.ugo_dot_attention.argtypes = [i64, i64, p, p, p, i64, p, i64, p, i64, ci, ci, ci, ctypes.c_double,
+                                          p, p, p]
+        lib.ugo_dot_attention.restype = ci
+        lib._dotattn_ready = True
+    src = _c32(src)
+    dst = _c32(dst)
+    E = int(src.shape[0])
+    q = np.ascontiguousarray(q, dtype=np.float32)
+    k = np.ascontiguousarray(k, dtype=np.float32)
+    val = np.ascontiguousarray(val, dtype=np.float32)
+    Dk = q.shape[1] // H
+    Dv = val.shape[1] // H
+    if scale is None:
+        scale = 1.0 / np.sqrt(Dk)
+    out = np.zeros((V, H * Dv), dtype=np.float64)
+    attn = np.zeros((max(E, 1), H), dtype=np.float64)
+    bnd = np.zeros((V, H * Dv), dtype=np.float64) if bound else None
+    rc = lib.ugo_dot_attention(V, E, _ptr(src), _ptr(dst), _ptr(q), q.shape[1], _ptr(k), k.shape[1],
+                               _ptr(val), val.shape[1], int(H), int(Dk), int(Dv), float(scale),
+                               _ptr(out), _ptr(attn), _ptr(bnd))
+    if rc != 0:
+        raise ValueError(f"oracle rejected dot_attention (H={H}) rc={rc}")
+    return (out, attn[:E], bnd) if bound else (out, attn[:E])
+
+
 def op_arg(V, src, dst, edge_op, gather_op, A=None, a_type=None, B=None, b_type=None, F=None, H=1):
     """Max/min aggregation with arg capture: returns (C [V, F] float32,
     arg [V, F] int64 edge ids, -1 for zero in-degree rows); ties keep the first edge id."""
