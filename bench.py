@@ -66,7 +66,8 @@ class ClockSampler:
     """nvidia-smi clocks / throttle reasons sampled every 50 ms during the timed region (the
     sampler's first row is awaited before the region starts, so short regions still get rows)."""
     Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap,power.draw,"
+         "enforced.power.limit")
 
     def __init__(self, index):
         self.index = index
@@ -91,7 +92,7 @@ class ClockSampler:
     def _read(self):
         for line in self.proc.stdout:
             parts = [x.strip() for x in line.split(",")]
-            if len(parts) == 6:
+            if len(parts) == 8:
                 self.rows.append(parts)
 
     def __exit__(self, *a):
@@ -109,11 +110,21 @@ class ClockSampler:
         mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = sorted({names[i] for r in self.rows for i in range(4) if r[2 + i] == "Active"})
+        def num(x):
+            try:
+                return float(x)
+            except ValueError:
+                return None
+        pw = [v for v in (num(r[6]) for r in self.rows) if v is not None]
+        lim = [v for v in (num(r[7]) for r in self.rows) if v is not None]
         out = {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-               "reasons": reasons, "samples": len(self.rows)}
+               "reasons": reasons, "samples": len(self.rows),
+               "power_w_median": round(statistics.median(pw), 1) if pw else None,
+               "power_w_max": round(max(pw), 1) if pw else None,
+               "enforced_power_limit_w": max(lim) if lim else None}
         if "sw_power_cap" in reasons:
-            out["note"] = ("sw_power_cap: the sustained L2-bound kernel runs at the board power limit, "
-                           "SM clock lowered by the driver (DESIGN.md 'Power')")
+            out["note"] = ("sw_power_cap: the sustained L2-bound kernel draws power_w_max against the "
+                           "enforced_power_limit_w; the driver lowers the SM clock (DESIGN.md 'Power')")
         return out
 
 
@@ -154,7 +165,66 @@ def oracle_sample(cfg_name, op, F, src, dst, V, target_s=15.0, seed=0):
 
 
 def cores_used():
+    """The oracle is single-threaded and this process is pinned to one core while it runs."""
     return 1
+
+
+def host_info():
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model}
+
+
+class PinnedCore:
+    """taskset -c 0 for the oracle timings: this process runs on core 0 only."""
+
+    def __enter__(self):
+        self.prev = os.sched_getaffinity(0)
+        os.sched_setaffinity(0, {min(self.prev)})
+        return self
+
+    def __exit__(self, *a):
+        os.sched_setaffinity(0, self.prev)
+
+
+def oracle_per_config(secondary):
+    """The oracle (1 pinned core) on every per_op_graph case of C1-C4 over the WHOLE graph, median
+    of 3 (SURVEY 8(d) / BASELINE.md 3), beside the GPU latency of the same op."""
+    import oracle
+    import ugdata
+    out = []
+    graphs = {}
+    for ent in secondary:
+        if "schedule" not in ent:
+            continue
+        cfg = ent["config"]
+        spec = next(x for x in SECONDARY if x[0] == cfg and x[1] == ent["op"] and x[7] == ent["F"])
+        _, nm, eo, go, a, b, c, F, H, wa, wb = spec
+        if cfg not in graphs:
+            graphs[cfg] = ugdata.graph(cfg)
+        src, dst = graphs[cfg]
+        V, E = ugdata.CONFIGS[cfg].V, len(src)
+        rows = lambda t: V if t in ("u", "v") else E
+        A = ugdata.values(rows(a), wa, 5, 1)
+        B = ugdata.values(rows(b), wb, 5, 2, role="den" if eo == "div" else "num") if b else None
+        ts = []
+        with PinnedCore():
+            for _ in range(3):
+                t0 = time.perf_counter()
+                oracle.op(V, src, dst, eo, go, A=A, a_type=a, B=B, b_type=b, c_type=c, F=F, H=H)
+                ts.append(time.perf_counter() - t0)
+        med = statistics.median(ts)
+        out.append({"config": cfg, "op": nm, "F": F, "H": H, "oracle_ms_median_of_3": round(med * 1e3, 3),
+                    "oracle_gbs": round(ent["logical_bytes"] / med / 1e9, 4),
+                    "gpu_us_warm": ent["warm"]["latency_us"],
+                    "gpu_over_oracle": round(med * 1e6 / ent["warm"]["latency_us"], 1)})
+    return out
 
 
 # Per op x graph latencies on the other BASELINE.json configs (C1-C4): (config, op name,
@@ -534,30 +604,44 @@ def main():
 
     traffic = None
     l2 = None
+    ncu_ent = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
         try:
-            ent = json.load(open(tp)).get(f"{args.config}:{args.op}:{F}:{chosen}")
+            ncu_ent = json.load(open(tp)).get(f"{args.config}:{args.op}:{F}:{chosen}")
             # dram__bytes_read.sum + dram__bytes_write.sum of one launch (ncu --set full)
-            traffic = int(ent["dram_bytes_per_launch"]) if ent and world == 1 else None
-            if ent and world == 1 and "l2_to_sm_bytes" in ent:
+            traffic = int(ncu_ent["dram_bytes_per_launch"]) if ncu_ent and world == 1 else None
+            if ncu_ent and world == 1 and "l2_to_sm_bytes" in ncu_ent:
                 # the binding roof of the tile-major schedule is L2 -> SM, not HBM
-                l2 = {"l2_to_sm_bytes_per_launch": int(ent["l2_to_sm_bytes"]),
-                      "achieved_gbs": round(ent["l2_to_sm_bytes"] / (kms * 1e-3) / 1e9, 1),
-                      "ncu_lts_throughput_pct": ent.get("lts_throughput_pct")}
+                l2 = {"l2_to_sm_bytes_per_launch": int(ncu_ent["l2_to_sm_bytes"]),
+                      "achieved_gbs": round(ncu_ent["l2_to_sm_bytes"] / (kms * 1e-3) / 1e9, 1),
+                      "ncu_lts_throughput_pct": ncu_ent.get("lts_throughput_pct"),
+                      "ncu_source": ncu_ent.get("source")}
         except (ValueError, OSError, KeyError, TypeError):
             traffic = None
 
     secondary = None
     if rank == 0 and world == 1 and not args.no_secondary:
         secondary = secondary_configs(ug, torch, dev)
+        # ncu DRAM bytes / L2 hit rate of the same (op, config, schedule), scripts/ncu_per_op.py
+        pp = os.path.join(ROOT, "profiles", "ncu_per_op.json")
+        if os.path.exists(pp):
+            prof = {(o["config"], o["op"], o["F"], o["schedule"]): o for o in json.load(open(pp))["ops"]}
+            for ent in secondary:
+                o = prof.get((ent.get("config"), ent.get("op"), ent.get("F"), ent.get("schedule")))
+                if o:
+                    ent["ncu"] = {"dram_bytes": o["dram_bytes"], "l2_to_sm_bytes": o["l2_to_sm_bytes"],
+                                  "l2_hit_rate_pct": o["l2_hit_rate_pct_main_kernel"], "cold_us": o["ncu_us"]}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        gbs, nr, ne, dt = oracle_sample(args.config, args.op, F, src, dst, V)
+        with PinnedCore():
+            gbs, nr, ne, dt = oracle_sample(args.config, args.op, F, src, dst, V)
         cpu = {"value": round(gbs, 4), "unit": "GB/s", "cores": cores_used(), "kind": "oracle",
                "sample": f"{args.op} on {nr} random dst rows ({ne} in-edges) of {args.config}, {dt:.1f} s, "
-                         f"oracle/ug_oracle.c single thread"}
+                         f"oracle/ug_oracle.c single thread pinned to one core (sched_setaffinity, = taskset -c 0)",
+               "host": host_info(),
+               "per_config": oracle_per_config(secondary) if secondary else None}
 
     if rank == 0:
         line = {
@@ -576,8 +660,15 @@ def main():
             **({"t_p": t_p} if t_p else {}),
             "graph_ingest_ms": round(ingest_ms, 1),
             "frac_of_8TBps": round(value / 8000.0, 4),
-            "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+            "roofline": {"bound": "l2" if l2 else "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": traffic,
+                         "frac_basis": ("logical (algorithmic, SURVEY 8(d)) bytes per live launch / measured HBM copy "
+                                        "bandwidth: an EFFECTIVE rate; above 1 because the tile-major SV schedule "
+                                        "serves the per-edge row gathers from L2. The binding roof is L2 -> SM: "
+                                        "l2_frac; DRAM use: dram_frac") if l2 else "algorithmic bytes / HBM peak",
+                         "l2_frac": round(l2["ncu_lts_throughput_pct"] / 100.0, 4)
+                                    if l2 and l2.get("ncu_lts_throughput_pct") else None,
+                         "dram_frac": round(traffic / (kms * 1e-3) / 1e9 / peak, 4) if traffic else None,
                          "kernel": ("k_split per 64-column chunk, exchange overlapped" if chunked else
                                     "k_split (SV main traversal)" if chosen.startswith("SV") else "main traversal"),
                          "kernel_ms": round(kms, 4), "peak_source": peak_src,

@@ -276,6 +276,23 @@ ug_status ug_gat_attention(const ug_graph *g, const float *el, int64_t ld_el, co
                            float slope, float *out, int64_t ld_out, float *attn, int64_t ld_attn,
                            void *stream);
 
+/* Fused dot-product attention chain (the FusedMM-style SDDMM + SpMM of
+ * PAPER.md:588 built from the paper's operators -- u_dot_v message creation (Table 2 dot ops,
+ * R5), an edge softmax over each destination's in-edges, and the u_mul_e_sum aggregation, the
+ * operator chain of PAPER.md:224 with a dot score) in ONE traversal:
+ *     s_e = scale * sum_{d<Dk} q[v][h*Dk+d] * k[u][h*Dk+d]      (e = u -> v, head h < H)
+ *     a_e = exp(s_e - max) / sum exp(... )  over the in-edges of v
+ *     out[v][h*Dv+j] = sum_e a_e * val[u][h*Dv+j]                 (0 for zero in-degree, R7)
+ *   q   [V][H*Dk] device, Dst_V rows (a view's local rows), row stride ld_q
+ *   k   [V_total][H*Dk], val [V_total][H*Dv] device, Src_V rows (global ids)
+ *   out [V][H*Dv] device (written); attn [E][H] device by edge id (written) or NULL.
+ *   Needs Dk and Dv <= 128 * vec where vec (4 / 2 / 1) divides both and every row's alignment;
+ *   else UG_ERR_SHAPE.  fp32 in / out; scores in the log2 domain with ex2.approx (R25).
+ *   Per-call scratch on `stream` (cudaMallocAsync): re-entrant across streams.  Asynchronous. */
+ug_status ug_dot_attention(const ug_graph *g, const float *q, int64_t ld_q, const float *k, int64_t ld_k,
+                           const float *val, int64_t ld_val, int32_t H, int32_t Dk, int32_t Dv, float scale,
+                           float *out, int64_t ld_out, float *attn, int64_t ld_attn, void *stream);
+
 /*
  * ug_op_run_arg -- a max/min aggregation with arg capture (training of
  * GraphSAGE-max style layers: the paper itself is inference-only).

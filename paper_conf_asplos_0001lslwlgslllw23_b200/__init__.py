@@ -20,7 +20,7 @@ from ._ffi import (EDGE_OPS, GATHER_OPS, STRATEGIES, TTYPES, UgError, UgOpInfo, 
                    UgTensor, check, lib)
 
 __all__ = ["Graph", "op_run", "prepare", "PreparedOp", "schedule_select", "launch_count", "parse_schedule",
-           "format_schedule", "validate", "edge_permute", "selector_load", "selector_load_model", "gat_attention", "op_run_arg", "arg_scatter", "reorder", "rows_gather", "Renumbered", "UgError",
+           "format_schedule", "validate", "edge_permute", "selector_load", "selector_load_model", "gat_attention", "dot_attention", "op_run_arg", "arg_scatter", "reorder", "rows_gather", "Renumbered", "UgError",
            "version"]
 
 
@@ -362,6 +362,37 @@ def gat_attention(graph, el, er, z, heads, slope=0.2, out=None, attn=None, strea
     pa, la = (None, 0) if attn is None else _mat(attn, "attn")
     check(lib.ug_gat_attention(graph.handle, pel, lel, per, ler, pz, lz, F, H, float(slope), po, lo, pa, la,
                                _current_stream(stream)), "ug_gat_attention")
+    return out
+
+
+def dot_attention(graph, q, k, val, heads, scale=None, out=None, attn=None, stream=None):
+    """Dot-product attention chain in ONE traversal (ug_dot_attention, the
+    FusedMM-style SDDMM + SpMM of PAPER.md:588 from the operators of PAPER.md:224):
+    out[v] = sum over in-edges e=(u->v) of softmax_e(scale * <q[v], k[u]>) per head * val[u].
+    q: [V, H*Dk] (Dst_V rows), k: [V_total, H*Dk], val: [V_total, H*Dv] (Src_V rows); scale
+    defaults to 1/sqrt(Dk).  Returns out [V, H*Dv] (and fills attn [E, H] if given)."""
+    import torch
+    H = int(heads)
+    Dk = int(q.shape[1]) // H
+    Dv = int(val.shape[1]) // H
+    if Dk * H != q.shape[1] or Dv * H != val.shape[1] or k.shape[1] != q.shape[1]:
+        raise ValueError("q / k widths must be H*Dk, val H*Dv")
+    vsrc, V, E = graph.dims()
+    if q.shape[0] < V or k.shape[0] < vsrc or val.shape[0] < vsrc:
+        raise ValueError("q needs one row per destination vertex, k / val one per source id")
+    if out is None:
+        out = torch.empty(V, H * Dv, device=val.device, dtype=torch.float32)
+    if scale is None:
+        scale = 1.0 / float(Dk) ** 0.5
+    pq, lq = _mat(q, "q")
+    pk, lk = _mat(k, "k")
+    pv, lv = _mat(val, "val")
+    po, lo = _mat(out, "out")
+    pa, la = (None, 0) if attn is None else _mat(attn, "attn")
+    if attn is not None and attn.shape[0] < E:
+        raise ValueError("attn needs one row per edge")
+    check(lib.ug_dot_attention(graph.handle, pq, lq, pk, lk, pv, lv, H, Dk, Dv, float(scale), po, lo, pa, la,
+                               _current_stream(stream)), "ug_dot_attention")
     return out
 
 

@@ -18,6 +18,9 @@ namespace ug {
 
 template <int GOP>
 __device__ __forceinline__ bool strictly_better(float m, float cur) {
+    // NaN is absorbing (R12): the first NaN message wins and stays
+    if (isnan(cur)) return false;
+    if (isnan(m)) return true;
     // before(x, y): x precedes y in the total order -0 < +0
     auto before = [](float x, float y) { return x < y || (x == y && signbit(x) && !signbit(y)); };
     return GOP == UG_GATHER_MAX ? before(cur, m) : before(m, cur);
@@ -73,7 +76,7 @@ __global__ void __launch_bounds__(256) k_argext(GraphArgs g, OpArgs op, int L_lo
     }
     if (ch.w < 0) {                                   // the row is one chunk
         if (active) {
-            op.C[v * op.c_ld + f] = be < 0 ? 0.0f : best;
+            op.C[v * op.c_ld + f] = be < 0 ? 0.0f : (isnan(best) ? __uint_as_float(UG_CANONICAL_NAN) : best);
             arg[v * ld_arg + f] = be;
         }
         return;
@@ -82,7 +85,7 @@ __global__ void __launch_bounds__(256) k_argext(GraphArgs g, OpArgs op, int L_lo
         sval[(int64_t)ch.w * sld + f] = best;
         sarg[(int64_t)ch.w * sld + f] = be;
     }
-    __threadfence();
+    fence_acq_rel_gpu();
     const unsigned smask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << (slice * L));
     __syncwarp(smask);
     const int r = slot_row[ch.w];
@@ -91,7 +94,7 @@ __global__ void __launch_bounds__(256) k_argext(GraphArgs g, OpArgs op, int L_lo
     if (sl == 0) last = atomicAdd(counters + (int64_t)r * n_tiles + tile, 1) == sp.z - 1;
     last = __shfl_sync(smask, last, slice * L);
     if (!last) return;
-    __threadfence();
+    fence_acq_rel_gpu();
     if (sl == 0) counters[(int64_t)r * n_tiles + tile] = 0;    // re-armed for the next call
     if (!active) return;
     best = 0.0f;
@@ -102,7 +105,7 @@ __global__ void __launch_bounds__(256) k_argext(GraphArgs g, OpArgs op, int L_lo
         const int32_t e = __ldcg(sarg + slot * sld + f);
         if (e >= 0 && (be < 0 || strictly_better<GOP>(m, best))) { best = m; be = e; }
     }
-    op.C[v * op.c_ld + f] = be < 0 ? 0.0f : best;
+    op.C[v * op.c_ld + f] = be < 0 ? 0.0f : (isnan(best) ? __uint_as_float(UG_CANONICAL_NAN) : best);
     arg[v * ld_arg + f] = be;
 }
 

@@ -23,17 +23,23 @@ __device__ __forceinline__ float edge_fn(float a, float b) {
 }
 
 // ---------------------------------------------------------------- gather_op (Fig. 5 line 19)
-// Total order with -0 < +0 (R12): fmaxf/fminf plus an explicit tie rule for +-0.
-__device__ __forceinline__ float tmax(float a, float b) {
-    float m = fmaxf(a, b);
-    if (a == b) m = __int_as_float(__float_as_int(a) & __float_as_int(b));
+// Total order with -0 < +0 and NaN-propagating (R12): max.NaN / min.NaN are IEEE 754-2019
+// maximum / minimum -- the canonical NaN 0x7FFFFFFF if either input is NaN, and -0 < +0 (measured
+// on this B200 by scripts/probes/minmax_zero.cu: max(-0, +0) = +0, min(-0, +0) = -0 in either
+// argument order), so no explicit signed-zero tie rule is needed.
+__device__ __forceinline__ float fmax_nan(float a, float b) {
+    float m;
+    asm("max.NaN.f32 %0, %1, %2;" : "=f"(m) : "f"(a), "f"(b));
     return m;
 }
-__device__ __forceinline__ float tmin(float a, float b) {
-    float m = fminf(a, b);
-    if (a == b) m = __int_as_float(__float_as_int(a) | __float_as_int(b));
+__device__ __forceinline__ float fmin_nan(float a, float b) {
+    float m;
+    asm("min.NaN.f32 %0, %1, %2;" : "=f"(m) : "f"(a), "f"(b));
     return m;
 }
+__device__ __forceinline__ float tmax(float a, float b) { return fmax_nan(a, b); }
+__device__ __forceinline__ float tmin(float a, float b) { return fmin_nan(a, b); }
+constexpr uint32_t UG_CANONICAL_NAN = 0x7FFFFFFFu;
 
 template <int GOP>
 __device__ __forceinline__ float g_init() {
@@ -296,12 +302,17 @@ __device__ __forceinline__ void gather_row(const GraphArgs &g, const OpArgs &op,
 // ---------------------------------------------------------------- atomics (pass 2)
 // max/min on fp32 by the integer-order trick: non-negative floats order like signed ints,
 // negative floats order reversed as unsigned ints; -0 (0x80000000) < +0 (0).
+// NaN (R12) is absorbing: for max it is stored as 0x7FFFFFFF (the largest positive int: no later
+// value replaces it); for min as 0xFFFFFFFF (the largest unsigned: no later value replaces it),
+// which the epilogue rewrites to the canonical 0x7FFFFFFF.
 __device__ __forceinline__ void atomic_max_f32(float *addr, float v) {
-    if (!signbit(v)) atomicMax(reinterpret_cast<int *>(addr), __float_as_int(v));
+    if (isnan(v)) atomicMax(reinterpret_cast<int *>(addr), (int)UG_CANONICAL_NAN);
+    else if (!signbit(v)) atomicMax(reinterpret_cast<int *>(addr), __float_as_int(v));
     else atomicMin(reinterpret_cast<unsigned int *>(addr), __float_as_uint(v));
 }
 __device__ __forceinline__ void atomic_min_f32(float *addr, float v) {
-    if (!signbit(v)) atomicMin(reinterpret_cast<int *>(addr), __float_as_int(v));
+    if (isnan(v)) atomicMax(reinterpret_cast<unsigned int *>(addr), 0xFFFFFFFFu);
+    else if (!signbit(v)) atomicMin(reinterpret_cast<int *>(addr), __float_as_int(v));
     else atomicMax(reinterpret_cast<unsigned int *>(addr), __float_as_uint(v));
 }
 
@@ -330,6 +341,11 @@ __device__ __forceinline__ void atomic_flush(float *p, const float (&acc)[VEC], 
         }
     }
 }
+
+// Release / acquire fence of the last-arriver merges (store partials; fence; relaxed atomicAdd
+// on the arrival counter  ||  atomicAdd; fence; load partials): the PTX fence-based
+// release-acquire pattern at gpu scope, lighter than __threadfence()'s fence.sc.gpu.
+__device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 
 // Helpers for launch sizing.
 __host__ __device__ __forceinline__ int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }

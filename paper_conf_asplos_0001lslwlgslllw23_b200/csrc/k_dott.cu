@@ -46,7 +46,7 @@ __device__ __forceinline__ float warp_sum8_transposed(float (&v)[8], int lane) {
 }
 
 #ifndef UG_DOTT_MINB
-#define UG_DOTT_MINB 4
+#define UG_DOTT_MINB 6
 #endif
 
 template <int VEC>
@@ -63,37 +63,47 @@ __global__ void __launch_bounds__(256, UG_DOTT_MINB) k_dott(GraphArgs g, OpArgs 
     const int o = ht / tiles_per_head, t = ht - o * tiles_per_head;
     const int fo = t * TW + lane * VEC;            // feature inside head o
     const bool active = fo < op.D;
-    const int f = o * op.D + (active ? fo : 0);
+    const int nval = active ? min(VEC, op.D - fo) : 0;   // < VEC only in a single head's ragged tail
+    const int f = o * op.D + (active ? fo : 0);   // inactive lanes load (and discard) a valid vector
     const Operand &P = a_is_src ? op.A : op.B;     // gathered per edge (Src_V)
     const Operand &Q = a_is_src ? op.B : op.A;     // hoisted (Dst_V, local row v)
     const int4 ch = chunks[c];
     const int64_t v = ch.x;
     const uint64_t keep = l2_policy_evict_last(), stream = l2_policy_evict_first();
     float q[VEC];
-    if (active) ldg_vec<VEC>(Q.p + v * Q.ld + f, q);
+    if (nval == VEC) ldg_vec<VEC>(Q.p + v * Q.ld + f, q);
     else
 #pragma unroll
-        for (int i = 0; i < VEC; ++i) q[i] = 0.0f;
+        for (int i = 0; i < VEC; ++i) q[i] = i < nval ? Q.p[v * Q.ld + f + i] : 0.0f;
     const float *__restrict__ Pb = P.p + f;
     const uint32_t ldp = (uint32_t)P.ld;
     float *dst = out + (int64_t)t * tile_stride + o;
     const int k1 = ch.z;
-    for (int k = ch.y; k < k1; k += 8) {
+    // a batch: 8 column indices, then 8 row gathers (UG_DOTT_PIPE=1 issues the next batch's before
+    // reducing the current one -- measured slower, kept for A/B)
+    auto load_batch = [&](int k, float (&x)[8][VEC]) {
         const int last = k1 - 1;
         uint32_t s[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) s[i] = (uint32_t)ldg_i32_hint(g.col + min(k + i, last), stream);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            // branch-free: every lane loads a full vector from a valid address (an inactive lane
+            // its head's first columns; a ragged tail reads into the packed row's padding) and
+            // zeroes the elements outside the head by select
+            ldg_vec_hint<VEC>(Pb + s[i] * ldp, x[i], keep);
+#pragma unroll
+            for (int j = 0; j < VEC; ++j) x[i][j] = j < nval ? x[i][j] : 0.0f;
+        }
+    };
+    float xa[8][VEC];
+    auto reduce_store = [&](int k, const float (&x)[8][VEC]) {
         float p[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
-            float x[VEC];
-            if (active) ldg_vec_hint<VEC>(Pb + s[i] * ldp, x, keep);
-            else
-#pragma unroll
-                for (int j = 0; j < VEC; ++j) x[j] = 0.0f;
             float a = 0.0f;
 #pragma unroll
-            for (int j = 0; j < VEC; ++j) a = __fmaf_rn(x[j], q[j], a);
+            for (int j = 0; j < VEC; ++j) a = __fmaf_rn(x[i][j], q[j], a);
             p[i] = a;
         }
         const float r = warp_sum8_transposed(p, lane);
@@ -101,6 +111,30 @@ __global__ void __launch_bounds__(256, UG_DOTT_MINB) k_dott(GraphArgs g, OpArgs 
         if ((lane & 3) == 0 && k + i < k1) {
             const int64_t e = g.eid ? (int64_t)g.eid[k + i] : (int64_t)(k + i);
             dst[e * out_ld] = r;
+        }
+    };
+    int k = ch.y;
+#ifndef UG_DOTT_PIPE
+#define UG_DOTT_PIPE 0
+#endif
+    if constexpr (!UG_DOTT_PIPE) {
+        // one batch in flight per warp: a second (software-pipelined) batch measured slower at every
+        // vector width (registers: 64 at VEC 2, spills at VEC 4; profiles/r2/ab_r2l.jsonl)
+        for (; k < k1; k += 8) {
+            load_batch(k, xa);
+            reduce_store(k, xa);
+        }
+    } else {
+        float xb[8][VEC];
+        if (k < k1) load_batch(k, xa);
+        while (k < k1) {
+            if (k + 8 < k1) load_batch(k + 8, xb);
+            reduce_store(k, xa);
+            k += 8;
+            if (k >= k1) break;
+            if (k + 8 < k1) load_batch(k + 8, xa);
+            reduce_store(k, xb);
+            k += 8;
         }
     }
 }

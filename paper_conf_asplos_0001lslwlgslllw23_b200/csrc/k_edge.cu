@@ -216,6 +216,7 @@ __global__ void k_epilogue(GraphArgs g, float *C, int64_t ld, int W, int mean) {
         float *p = C + v * ld + (i - v * W);
         if (deg == 0) *p = 0.0f;
         else if (mean) *p = __fdiv_rn(*p, (float)deg);
+        else if (isnan(*p)) *p = __uint_as_float(UG_CANONICAL_NAN);   // min's 0xFFFFFFFF (R12)
     }
 }
 

@@ -184,7 +184,7 @@ __global__ void __launch_bounds__(256) k_gat(GraphArgs g, GatArgs a, int L_log2,
         sst[((int64_t)ch.w * 2) * nfc + fc] = st.m;
         sst[((int64_t)ch.w * 2 + 1) * nfc + fc] = st.den;
     }
-    __threadfence();
+    fence_acq_rel_gpu();
     const unsigned smask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << (slice * L));
     __syncwarp(smask);
     const int r = slot_row[ch.w];
@@ -193,7 +193,7 @@ __global__ void __launch_bounds__(256) k_gat(GraphArgs g, GatArgs a, int L_log2,
     if (sl == 0) last = atomicAdd(counters + (int64_t)r * n_tiles + tile, 1) == sp.z - 1;
     last = __shfl_sync(smask, last, slice * L);
     if (!last) return;
-    __threadfence();
+    fence_acq_rel_gpu();
     if (sl == 0) counters[(int64_t)r * n_tiles + tile] = 0;    // re-armed for the next call
     st.init();
     for (int i = 0; i < sp.z; ++i) {

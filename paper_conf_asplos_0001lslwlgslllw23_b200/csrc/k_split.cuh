@@ -246,21 +246,91 @@ __device__ __forceinline__ int unit_tile(int64_t u, int64_t n_chunks, int n_tile
     return u < INT32_MAX ? (int)((uint32_t)u / (uint32_t)n_chunks) : (int)(u / n_chunks);
 }
 
-template <int KE, int GOP, int VEC, int BM>
+// Single-launch merge of a split row: every chunk of the row has stored its partial; the unit
+// that arrives last (per row and column tile) combines the partials in chunk order -- the order
+// k_split_fix uses, so results are identical -- and re-arms the counter for the next call on
+// this stream.  Called by every lane of a unit whose chunk belongs to a split row.
+template <int GOP, int VEC>
+__device__ __forceinline__ void split_merge(const GraphArgs &g, const OpArgs &op, const int4 *__restrict__ chunks,
+                                            const int64_t n_chunks, const int L_log2, const int ftile,
+                                            const int n_tiles, const float *__restrict__ scratch, const int64_t sld,
+                                            const int4 *__restrict__ split, const int32_t *__restrict__ slot_row,
+                                            int32_t *__restrict__ counters) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int L = 1 << L_log2;
+    const int lane = (int)(t & (L - 1));
+    const int64_t u = t >> L_log2;
+    const int tile = unit_tile(u, n_chunks, n_tiles);
+    const int f = tile * ftile + lane * VEC;
+    int4 ch;   // re-read (volatile: not kept live from the traversal)
+    asm volatile("ld.global.cg.v4.s32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(ch.x), "=r"(ch.y), "=r"(ch.z), "=r"(ch.w) : "l"(chunks + (u - (int64_t)tile * n_chunks)));
+    if (ch.w < 0) return;                         // an owned row: finished in the traversal
+    fence_acq_rel_gpu();
+    const int wl = threadIdx.x & 31;
+    const unsigned umask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << (wl & ~(L - 1)));
+    __syncwarp(umask);
+    const int r = slot_row[ch.w];
+    const int4 sp = split[r];
+    int last = 0;
+    if (lane == 0) last = atomicAdd(counters + (int64_t)r * n_tiles + tile, 1) == sp.z - 1;
+    last = __shfl_sync(umask, last, wl & ~(L - 1));
+    if (!last) return;
+    fence_acq_rel_gpu();
+    if (lane == 0) counters[(int64_t)r * n_tiles + tile] = 0;
+    if (f >= op.W) return;
+    float acc[VEC];
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) acc[i] = g_init<GOP>();
+    for (int c = 0; c < sp.z; ++c) {
+        const float *pp = scratch + (int64_t)(sp.y + c) * sld + f;
+        float p[VEC];
+        if constexpr (VEC == 4) {
+            const float4 x = __ldcg(reinterpret_cast<const float4 *>(pp));
+            p[0] = x.x; p[1] = x.y; p[2] = x.z; p[3] = x.w;
+        } else if constexpr (VEC == 2) {
+            const float2 x = __ldcg(reinterpret_cast<const float2 *>(pp));
+            p[0] = x.x; p[1] = x.y;
+        } else {
+            p[0] = __ldcg(pp);
+        }
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) acc[i] = g_combine<GOP>(acc[i], p[i]);
+    }
+    const int64_t v = sp.x;
+    const int64_t deg = (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) acc[i] = g_finalize<GOP>(acc[i], deg);
+    st_out<VEC>(op.C + v * op.c_ld + f, acc, op.W - f, op.c_vec);
+}
+
+template <int KE, int GOP, int VEC, int BM, bool MERGE>
 #ifndef UG_ASSIGN_MINB
 #define UG_ASSIGN_MINB 6
 #endif
 __global__ void __launch_bounds__(256, (UG_ASSIGN_MINB > 0 && GOP == UG_GATHER_ASSIGN) ? UG_ASSIGN_MINB : (BM == 0) ? UG_BM0_MINB : (BM == 2 ? ((GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN) && KE != K_DIV ? UG_BM2_SUM_MINB : UG_BM2_MINB) : (BM > 0 ? (VEC == 4 ? 5 : 6) : 4))) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
                                                int64_t n_chunks, int L_log2, int ftile, int n_tiles,
-                                               float *__restrict__ scratch, int64_t sld) {
+                                               float *__restrict__ scratch, int64_t sld,
+                                               const int4 *__restrict__ split, const int32_t *__restrict__ slot_row,
+                                               int32_t *__restrict__ counters) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int lane = (int)(t & ((1 << L_log2) - 1));
     const int64_t u = t >> L_log2;
-    if (u >= n_chunks * n_tiles) return;
+    if (u >= n_chunks * n_tiles) return;          // whole units only: a unit's L lanes leave together
     const int tile = unit_tile(u, n_chunks, n_tiles);
     const int f = tile * ftile + lane * VEC;
-    if (f >= op.W) return;
-    split_unit<KE, GOP, VEC, BM>(g, op, chunks[u - (int64_t)tile * n_chunks], f, scratch, sld);
+    if constexpr (!MERGE) {
+        // split rows (if any) are combined by k_split_fix, a second launch
+        if (f >= op.W) return;
+        split_unit<KE, GOP, VEC, BM>(g, op, chunks[u - (int64_t)tile * n_chunks], f, scratch, sld);
+    } else {
+        // single-launch merge of split rows: the last-arriving chunk of a row combines them.  A
+        // separate instance (launch-bound small graphs): the merge needs every lane of the unit
+        // and re-derives its indices after the in-edge loop.
+        if (f < op.W) split_unit<KE, GOP, VEC, BM>(g, op, chunks[u - (int64_t)tile * n_chunks], f, scratch, sld);
+        split_merge<GOP, VEC>(g, op, chunks, n_chunks, L_log2, ftile, n_tiles, scratch, sld, split, slot_row,
+                              counters);
+    }
 }
 
 // Fix-up of split rows: combine the row's partials in chunk order, finalise, store.
@@ -293,7 +363,7 @@ __global__ void k_split_fix(GraphArgs g, OpArgs op, const int4 *__restrict__ spl
 template <int KE>
 cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, const LaunchCfg &c,
                             const SplitPlan &plan, float *scratch, cudaStream_t s, cudaEvent_t ev_begin,
-                            cudaEvent_t ev_end) {
+                            cudaEvent_t ev_end, int32_t *counters) {
     const int L = c.ftile / c.vec;
     const int n_tiles = (int)cdiv(op.W, c.ftile);
     const int64_t threads = plan.n_chunks * n_tiles * (int64_t)L;
@@ -302,6 +372,8 @@ cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, co
     const int L_log2 = ilog2(L);
     const int64_t sld = cdiv(op.W, 4) * 4;
     const int4 *chunks = reinterpret_cast<const int4 *>(plan.d_chunk);
+    const int4 *split_p = reinterpret_cast<const int4 *>(plan.d_split);
+    if (plan.n_split_rows == 0 || gather == UG_GATHER_ASSIGN) counters = nullptr;
     if (ev_begin) cudaEventRecord(ev_begin, s);
     // fast path: full-width Src_V A operand, identity edge ids, and every operand row
     // addressable with 32-bit element offsets (rows * ld < 2^32)
@@ -315,9 +387,20 @@ cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, co
     const int bfl = op.B.div == 1 ? 1 : 0;
     const int bm = !fast ? -1 : KE == K_COPY ? 0
                  : op.B.type == UG_T_DST_V ? 1 : (op.B.type == UG_T_EDGE ? 2 + bfl : 4 + bfl);
-#define UG_SV_LAUNCH(BMV)                                                                               \
-    k_split<KE, GOP, VEC, BMV><<<(unsigned)grid, c.block, 0, s>>>(g, op, chunks, plan.n_chunks, L_log2, \
-                                                                 c.ftile, n_tiles, scratch, sld)
+#define UG_SV_LAUNCH(BMV)                                                                                    \
+    do {                                                                                                     \
+        if constexpr (GOP != UG_GATHER_ASSIGN) {                                                             \
+            if (counters) {                                                                                  \
+                k_split<KE, GOP, VEC, BMV, true><<<(unsigned)grid, c.block, 0, s>>>(                         \
+                    g, op, chunks, plan.n_chunks, L_log2, c.ftile, n_tiles, scratch, sld, split_p,           \
+                    plan.d_slot_row, counters);                                                              \
+                break;                                                                                       \
+            }                                                                                                \
+        }                                                                                                    \
+        k_split<KE, GOP, VEC, BMV, false><<<(unsigned)grid, c.block, 0, s>>>(                                \
+            g, op, chunks, plan.n_chunks, L_log2, c.ftile, n_tiles, scratch, sld, split_p, plan.d_slot_row,   \
+            nullptr);                                                                                        \
+    } while (0)
     UG_DISPATCH_VEC(c.vec, VEC,
         UG_DISPATCH_GOP(gather, GOP, {
             if constexpr (KE == K_COPY) {
@@ -336,7 +419,7 @@ cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, co
 #undef UG_SV_LAUNCH
     if (ev_end) cudaEventRecord(ev_end, s);
     cudaError_t err = cudaGetLastError();
-    if (err != cudaSuccess || gather == UG_GATHER_ASSIGN || plan.n_split_rows == 0) return err;
+    if (err != cudaSuccess || gather == UG_GATHER_ASSIGN || plan.n_split_rows == 0 || counters) return err;
     const int64_t per_row = cdiv(op.W, c.vec);
     const int64_t fgrid = cdiv(plan.n_split_rows * per_row, 256);
     const int4 *split = reinterpret_cast<const int4 *>(plan.d_split);
@@ -350,6 +433,6 @@ cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, co
 #define UG_SV_INSTANTIATE(KE)                                                                            \
     template cudaError_t launch_split_ke<KE>(int, const GraphArgs &, const OpArgs &, const LaunchCfg &, \
                                              const SplitPlan &, float *, cudaStream_t, cudaEvent_t,     \
-                                             cudaEvent_t);
+                                             cudaEvent_t, int32_t *);
 
 }  // namespace ug

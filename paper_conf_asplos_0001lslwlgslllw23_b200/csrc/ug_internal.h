@@ -6,6 +6,7 @@
 #include <map>
 #include <mutex>
 #include <string>
+#include <tuple>
 #include <vector>
 
 #include "ug.h"
@@ -79,7 +80,8 @@ cudaError_t launch_block_vertex(int kedge, int gather, const GraphArgs &g, const
                                 const LaunchCfg &c, cudaStream_t s);
 cudaError_t launch_split_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
                                 const LaunchCfg &c, const SplitPlan &plan, float *scratch,
-                                cudaStream_t s, cudaEvent_t ev_begin = nullptr, cudaEvent_t ev_end = nullptr);
+                                cudaStream_t s, cudaEvent_t ev_begin = nullptr, cudaEvent_t ev_end = nullptr,
+                                int32_t *counters = nullptr);
 // SV with shared-memory row staging (k_svg.cu): mode 0 TMA gather4, 1 cp.async; bm = B addressing
 // mode (0 none, 1 Dst_V, 2 Edge broadcast).
 bool svg_supported(const OpArgs &op, int vec, int mode);
@@ -112,6 +114,19 @@ struct GatArgs {
 cudaError_t launch_gat(const GraphArgs &g, const GatArgs &a, int vec, int L, const SplitPlan &plan,
                        const int32_t *slot_row, float *sacc, float *sst, int64_t sld, int64_t nfc,
                        int32_t *counters, cudaStream_t s);
+// Fused dot-product attention chain (ug_dot_attention, k_dotattn.cu).
+struct DotAttnArgs {
+    const float *q, *k, *val;      // q: Dst_V [V][H*Dk] (local rows), k / val: Src_V [V_src][H*Dk / H*Dv]
+    int64_t ld_q, ld_k, ld_val;
+    float *out, *attn;             // out [V][H*Dv] (local rows); attn [E][H] by edge id or NULL
+    int64_t ld_out, ld_attn;
+    float *mden;                   // [V][H][2] final (max, denominator) per row and head (attn only)
+    int32_t H, Dk, Dv;
+    float scale_log2;              // scale * log2(e)
+};
+int dotattn_vec(const DotAttnArgs &a);
+cudaError_t launch_dotattn(const GraphArgs &g, const DotAttnArgs &a, int vec, const SplitPlan &plan,
+                           float *scratch, int64_t sld, cudaStream_t s);
 cudaError_t launch_argext(int kedge, int gather, const GraphArgs &g, const OpArgs &op, int L, const SplitPlan &plan,
                           const int32_t *slot_row, float *sval, int32_t *sarg, int64_t sld, int32_t *counters,
                           int32_t *arg, int64_t ld_arg, cudaStream_t s);
@@ -156,6 +171,10 @@ struct ug_graph {
     // UG_SV plans keyed by chunk size.
     mutable std::mutex mu;
     mutable std::map<int, ug::SplitPlan> plans;
+    // arrival counters of single-launch split-row merges (k_split, k_gat, k_argext), one buffer per
+    // (stream, chunk size, column tiles): n_split_rows x n_tiles int32, zeroed once; every call
+    // leaves them zero again, and calls on one stream are ordered, so no two calls share them
+    mutable std::map<std::tuple<void *, int, int>, int32_t *> stream_counters;
     // src vertex by edge id (device), built on first use when eid is not the identity
     mutable int32_t *d_src_of_eid = nullptr;
     mutable std::vector<void *> plan_allocs;

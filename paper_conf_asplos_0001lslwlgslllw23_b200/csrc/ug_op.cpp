@@ -3,6 +3,7 @@
 // PAPER.md:291-307; Table 2), lowering (the paper's two code-generation
 // passes, done as template selection), schedule resolution and launch.
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <algorithm>
 #include <cstdio>
@@ -178,25 +179,28 @@ ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, La
         *cfg = c;
         return UG_OK;
     }
-    if (c.strategy == UG_SV && lw.dot && s.ftile > 0) {
-        // k_dott: column tiles of 32 * vec features of each head, any D (ftile = the widest tile)
+    const bool dott_pair = lw.dot && lw.args.A.div == 1 && lw.args.B.div == 1 &&
+                           ((lw.args.A.type == UG_T_SRC_V && lw.args.B.type == UG_T_DST_V) ||
+                            (lw.args.A.type == UG_T_DST_V && lw.args.B.type == UG_T_SRC_V));
+    if (c.strategy == UG_SV && dott_pair && (s.ftile == 32 || s.ftile == 64 || s.ftile == 128)) {
+        // k_dott: column tiles of 32 * vec features of each head, any D (ftile = the widest tile);
+        // other ftile values, and dot ops that are not (Src_V, Dst_V) pairs, keep the untiled SV
+        // dot kernels (k_dotsv / k_dot), which ignore ftile
         const Operand &A = lw.args.A, &B = lw.args.B;
         const bool as = A.type == UG_T_SRC_V && B.type == UG_T_DST_V;
-        const bool bs = A.type == UG_T_DST_V && B.type == UG_T_SRC_V;
-        if (!(as || bs) || A.div != 1 || B.div != 1)
-            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "SV dot with ftile: one full-width Src_V and one Dst_V operand");
-        if (s.ftile != 32 && s.ftile != 64 && s.ftile != 128)
-            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "SV dot: ftile must be 32, 64 or 128");
         const Operand &P = as ? A : B, &Q = as ? B : A;
         auto fits = [&](const Operand &o, int v) { return (uintptr_t)o.p % (4 * v) == 0 && o.ld % v == 0; };
         const bool same = P.p == Q.p && P.ld == Q.ld;          // u_dot_v of one matrix with itself
         c.pack = false;
         int v = s.ftile / 32;
-        // widest v <= ftile / 32 with D % v == 0 and Q's rows aligned for v (P is packed into
-        // 128-byte rows when its own rows are not; a Q that is the same matrix follows it)
+        // widest v <= ftile / 32 with D % v == 0 (one head: any D) and Q's rows aligned for v (P is
+        // packed into 128-byte rows when its own rows are not; a Q that is the same matrix
+        // follows it).  A ragged head tail (D % v != 0) is gathered as a full vector and masked,
+        // so P's rows must reach round_up(D, v) -- packing guarantees it; Q, loaded once per
+        // unit, reads its tail element by element.
         for (; v > 1; v >>= 1)
-            if (lw.args.D % v == 0 && (fits(Q, v) || same)) break;
-        if (v > 1 && !fits(P, v)) c.pack = true;
+            if ((lw.args.D % v == 0 || lw.args.H == 1) && (fits(Q, v) || same)) break;
+        if (v > 1 && (!fits(P, v) || (lw.args.D % v != 0 && P.ld < (lw.args.D + v - 1) / v * v))) c.pack = true;
         if (s.vec && s.vec != v) return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "SV dot: vec follows ftile and the layout");
         c.dott = true;
         c.vec = v;
@@ -335,7 +339,34 @@ static ug_status get_plan(const ug_graph *g, int G, const SplitPlan **out) {
     return UG_OK;
 }
 
-static int launches_for(const Lowered &lw, const LaunchCfg &c, int64_t n_split_rows) {
+// Arrival counters of the single-launch split-row merges for calls on `stream` (see ug_graph::
+// stream_counters).  Allocated and zeroed once per (stream, chunk size, column tiles), in relaxed
+// capture mode like the plans; calls on one stream are ordered, and each call re-arms the counters
+// it used, so concurrent calls on different streams never share a counter.
+static ug_status get_counters(const ug_graph *g, void *stream, int G, int n_tiles, int64_t n_split_rows,
+                              int32_t **out) {
+    std::lock_guard<std::mutex> lock(g->mu);
+    const auto key = std::make_tuple(stream, G, n_tiles);
+    auto it = g->stream_counters.find(key);
+    if (it != g->stream_counters.end()) { *out = it->second; return UG_OK; }
+    RelaxedCapture relaxed;
+    void *d = nullptr;
+    const size_t bytes = std::max<size_t>(16, (size_t)n_split_rows * (size_t)n_tiles * 4);
+    if (cudaMalloc(&d, bytes) != cudaSuccess) return set_error(UG_ERR_OOM, "counter allocation failed");
+    g->plan_allocs.push_back(d);
+    if (cudaMemset(d, 0, bytes) != cudaSuccess) return set_error(UG_ERR_CUDA, "counter init failed");
+    g->stream_counters.emplace(key, (int32_t *)d);
+    *out = (int32_t *)d;
+    return UG_OK;
+}
+
+// Operators small enough to be launch-bound (per-edge feature work below ~2^26 elements) merge
+// split rows inside the traversal launch (k_split<..., MERGE>).
+static bool sv_merge_ok(const ug_graph *g, const Lowered &lw) {
+    return (double)g->E * (double)lw.args.W < 67108864.0;
+}
+
+static int launches_for(const ug_graph *g, const Lowered &lw, const LaunchCfg &c, int64_t n_split_rows) {
     if (c.dott) {
         const int msg = 1 + (dott_tiles(lw.args, c.vec) > 1 ? 1 : 0);
         return lw.to_edges ? msg : msg + (n_split_rows > 0 ? 2 : 1);
@@ -343,6 +374,7 @@ static int launches_for(const Lowered &lw, const LaunchCfg &c, int64_t n_split_r
     const bool edge_units = c.strategy == UG_TE || c.strategy == UG_WE || c.strategy == UG_BE;
     if (lw.to_edges) return 1;
     if (edge_units) return lw.gather == UG_GATHER_SUM ? 2 : 3;
+    if (c.strategy == UG_SV && !lw.dot && !c.staged && sv_merge_ok(g, lw)) return 1;   // merged in the launch
     if (c.strategy == UG_SV && (!lw.dot || dotsv_ok(lw, c))) return n_split_rows > 0 ? 2 : 1;
     return 1;
 }
@@ -391,7 +423,7 @@ extern "C" ug_status ug_op_launch_count(const ug_graph *g, const ug_op_info *op,
         for (int64_t v = 0; v < g->V; ++v)
             if ((int64_t)g->h_row_ptr[v + 1] - g->h_row_ptr[v] > c.G) ++nsr;
     }
-    *launches = launches_for(lw, c, nsr);
+    *launches = launches_for(g, lw, c, nsr);
     return UG_OK;
 }
 
@@ -555,7 +587,19 @@ static ug_status run(const ug_graph *g, const ug_op_info *op, const ug_schedule 
             err = launch_split_staged(mode, lw.kedge, lw.gather, ga, args, c.vec, bm, *plan, scratch, s, ev_begin,
                                       ev_end);
         } else {
-            err = launch_split_vertex(lw.kedge, lw.gather, ga, args, c, *plan, scratch, s, ev_begin, ev_end);
+            // single-launch merge of split rows for launch-bound (small) operators; large ones keep
+            // the hot instance without the merge tail and fix split rows in a second launch (< 1 %)
+            int32_t *counters = nullptr;
+            if (agg && plan->n_split_rows > 0 && sv_merge_ok(g, lw)) {
+                const int n_tiles = (int)((lw.args.W + c.ftile - 1) / c.ftile);
+                if ((st = get_counters(g, stream, c.G, n_tiles, plan->n_split_rows, &counters)) != UG_OK) {
+                    if (scratch) cudaFreeAsync(scratch, s);
+                    if (packed) cudaFreeAsync(packed, s);
+                    return st;
+                }
+            }
+            err = launch_split_vertex(lw.kedge, lw.gather, ga, args, c, *plan, scratch, s, ev_begin, ev_end,
+                                      counters);
         }
         if (scratch) cudaFreeAsync(scratch, s);
         if (packed) cudaFreeAsync(packed, s);
@@ -564,12 +608,21 @@ static ug_status run(const ug_graph *g, const ug_op_info *op, const ug_schedule 
     return UG_OK;
 }
 
+// One NVTX range per operator call (per-op ranges for nsys / ncu --nvtx); NVTX v3 is
+// header-only and costs a branch when no tool is attached.
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
+
 extern "C" ug_status ug_op_run(const ug_graph *g, const ug_op_info *op, const ug_schedule *sched, void *stream) {
+    NvtxRange r("ug_op_run");
     return run(g, op, sched, stream, nullptr, nullptr);
 }
 
 extern "C" ug_status ug_op_run_events(const ug_graph *g, const ug_op_info *op, const ug_schedule *sched,
                                       void *stream, void *ev_begin, void *ev_end) {
+    NvtxRange r("ug_op_run");
     return run(g, op, sched, stream, (cudaEvent_t)ev_begin, (cudaEvent_t)ev_end);
 }
 
@@ -698,27 +751,71 @@ extern "C" ug_status ug_gat_attention(const ug_graph *g, const float *el, int64_
     a.F = F; a.H = H; a.D = D; a.slope = slope;
     cudaStream_t s = (cudaStream_t)stream;
     const int64_t sld = (F + 3) / 4 * 4, nfc = (F + vec - 1) / vec;
-    // split-row partials, then the per-call arrival counters of the last-arriver merge (one per
-    // (split row, column tile), zeroed on this stream): calls on other streams never share them
+    // split-row partials (per call, stream-ordered) and this stream's arrival counters
     float *scratch = nullptr;
     int32_t *counters = nullptr;
     if (plan->n_split_chunks > 0) {
+        if ((st = get_counters(g, stream, G, n_tiles, plan->n_split_rows, &counters)) != UG_OK) return st;
         ensure_pool_retains();
         const size_t part = sizeof(float) * (size_t)plan->n_split_chunks * (size_t)(sld + 2 * nfc);
-        const size_t cnt = sizeof(int32_t) * (size_t)plan->n_split_rows * (size_t)n_tiles;
-        if (cudaMallocAsync((void **)&scratch, part + cnt, s) != cudaSuccess)
+        if (cudaMallocAsync((void **)&scratch, part, s) != cudaSuccess)
             return set_error(UG_ERR_OOM, "ug_gat_attention: scratch allocation failed");
-        counters = reinterpret_cast<int32_t *>(reinterpret_cast<char *>(scratch) + part);
-        if (cudaMemsetAsync(counters, 0, cnt, s) != cudaSuccess) {
-            cudaFreeAsync(scratch, s);
-            return set_error(UG_ERR_CUDA, "ug_gat_attention: counter init failed");
-        }
     }
     float *sst = scratch ? scratch + plan->n_split_chunks * sld : nullptr;
     cudaError_t e = launch_gat(graph_args(g), a, vec, L, *plan, plan->d_slot_row, scratch, sst, sld, nfc,
                                counters, s);
     if (scratch) cudaFreeAsync(scratch, s);
     if (e != cudaSuccess) return set_error(UG_ERR_CUDA, std::string("ug_gat_attention: ") + cudaGetErrorString(e));
+    return UG_OK;
+}
+
+// ------------------------------------------------------------------------- fused dot attention (f3)
+extern "C" ug_status ug_dot_attention(const ug_graph *g, const float *q, int64_t ld_q, const float *k, int64_t ld_k,
+                                      const float *val, int64_t ld_val, int32_t H, int32_t Dk, int32_t Dv,
+                                      float scale, float *out, int64_t ld_out, float *attn, int64_t ld_attn,
+                                      void *stream) {
+    using namespace ug;
+    if (!g) return set_error(UG_ERR_INVALID_ARG, "ug_dot_attention: NULL graph");
+    if (g->host_only) return set_error(UG_ERR_INVALID_ARG, "ug_dot_attention needs a device graph");
+    if (H <= 0 || Dk <= 0 || Dv <= 0) return set_error(UG_ERR_SHAPE, "ug_dot_attention: need H, Dk, Dv > 0");
+    if (ld_q < (int64_t)H * Dk || ld_k < (int64_t)H * Dk || ld_val < (int64_t)H * Dv || ld_out < (int64_t)H * Dv ||
+        (attn && ld_attn < H))
+        return set_error(UG_ERR_SHAPE, "ug_dot_attention: ld < width");
+    if (g->V > 0 && (!q || !out)) return set_error(UG_ERR_INVALID_ARG, "ug_dot_attention: NULL q / out");
+    if (g->E > 0 && (!k || !val)) return set_error(UG_ERR_INVALID_ARG, "ug_dot_attention: NULL k / val");
+    if (g->V == 0) return UG_OK;
+    DotAttnArgs a;
+    a.q = q; a.k = k; a.val = val;
+    a.ld_q = ld_q; a.ld_k = ld_k; a.ld_val = ld_val;
+    a.out = out; a.attn = attn; a.ld_out = ld_out; a.ld_attn = ld_attn;
+    a.mden = nullptr;
+    a.H = H; a.Dk = Dk; a.Dv = Dv;
+    a.scale_log2 = scale * 1.4426950408889634f;
+    const int vec = dotattn_vec(a);
+    if (vec == 0) return set_error(UG_ERR_SHAPE, "ug_dot_attention: Dk and Dv must be <= 128 * vec (vec 4 / 2 / 1)");
+    if ((uint64_t)g->V_total * (uint64_t)std::max(ld_k, ld_val) >= (1ull << 32))
+        return set_error(UG_ERR_SHAPE, "ug_dot_attention: k / val above 2^32 elements");
+    int G = 64;
+    if (const char *ev = std::getenv("UG_DOTATTN_CHUNK")) G = std::max(1, std::atoi(ev));
+    const SplitPlan *plan = nullptr;
+    ug_status st = get_plan(g, G, &plan);
+    if (st != UG_OK) return st;
+    if (plan->n_chunks * (int64_t)H >= ((int64_t)1 << 31) - 8)
+        return set_error(UG_ERR_SHAPE, "ug_dot_attention: more than 2^31 (chunk, head) units");
+    cudaStream_t s = (cudaStream_t)stream;
+    const int64_t sld = ((int64_t)Dv + 4 + 3) / 4 * 4;
+    const size_t part = sizeof(float) * (size_t)plan->n_split_chunks * (size_t)H * (size_t)sld;
+    const size_t md = attn ? sizeof(float) * (size_t)g->V * (size_t)H * 2 : 0;
+    float *scratch = nullptr;
+    if (part + md > 0) {
+        ensure_pool_retains();
+        if (cudaMallocAsync((void **)&scratch, part + md, s) != cudaSuccess)
+            return set_error(UG_ERR_OOM, "ug_dot_attention: scratch allocation failed");
+        if (attn) a.mden = reinterpret_cast<float *>(reinterpret_cast<char *>(scratch) + part);
+    }
+    cudaError_t e = launch_dotattn(graph_args(g), a, vec, *plan, scratch, sld, s);
+    if (scratch) cudaFreeAsync(scratch, s);
+    if (e != cudaSuccess) return set_error(UG_ERR_CUDA, std::string("ug_dot_attention: ") + cudaGetErrorString(e));
     return UG_OK;
 }
 
@@ -749,17 +846,11 @@ extern "C" ug_status ug_op_run_arg(const ug_graph *g, const ug_op_info *op, int3
     float *scratch = nullptr;
     int32_t *counters = nullptr;
     if (plan->n_split_chunks > 0) {
-        // partial values + partial args, then per-call arrival counters zeroed on this stream
+        // partial values + partial args (per call, stream-ordered); this stream's arrival counters
+        if ((st = get_counters(g, stream, G, n_tiles, plan->n_split_rows, &counters)) != UG_OK) return st;
         ensure_pool_retains();
-        const size_t part = (size_t)plan->n_split_chunks * sld * 8;
-        const size_t cnt = sizeof(int32_t) * (size_t)plan->n_split_rows * (size_t)n_tiles;
-        if (cudaMallocAsync((void **)&scratch, part + cnt, s) != cudaSuccess)
+        if (cudaMallocAsync((void **)&scratch, (size_t)plan->n_split_chunks * sld * 8, s) != cudaSuccess)
             return set_error(UG_ERR_OOM, "ug_op_run_arg: scratch allocation failed");
-        counters = reinterpret_cast<int32_t *>(reinterpret_cast<char *>(scratch) + part);
-        if (cudaMemsetAsync(counters, 0, cnt, s) != cudaSuccess) {
-            cudaFreeAsync(scratch, s);
-            return set_error(UG_ERR_CUDA, "ug_op_run_arg: counter init failed");
-        }
     }
     int32_t *sarg = scratch ? reinterpret_cast<int32_t *>(scratch + plan->n_split_chunks * sld) : nullptr;
     cudaError_t e = launch_argext(lw.kedge, lw.gather, graph_args(g), lw.args, L, *plan, plan->d_slot_row, scratch,

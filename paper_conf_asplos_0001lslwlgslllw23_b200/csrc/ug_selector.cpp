@@ -214,7 +214,9 @@ static bool model_select(const ug_graph *g, const Lowered &lw, ug_schedule *out)
 // width (measured with float4 rows, applied to float2 rows): keep 32 lanes.
 static ug_schedule adapt(const Lowered &lw, ug_schedule s) {
     if (s.vec > lw.max_vec) s.vec = 0;
-    if (s.strategy == UG_SV && s.ftile > 0) {
+    // (dot under SV with a column tile is k_dott, which picks its own vector width and packs P;
+    // staged SV fixes vec = ftile / 32 itself)
+    if (s.strategy == UG_SV && s.ftile > 0 && !lw.dot && !(s.flags & (UG_SCHED_TMA | UG_SCHED_ASYNC))) {
         const bool pack = (s.flags & UG_SCHED_PACK) && lw.pack_ok;
         const int vec = std::max(1, std::min(pack ? 4 : lw.a_vec, lw.b_vec));
         if (s.ftile / vec > 32 || s.ftile % vec) s.ftile = 32 * vec;

@@ -83,6 +83,32 @@ def full(path):
     return res
 
 
+def traffic(path, key, out="profiles/ncu_traffic.json"):
+    """Add the bench kernel's per-launch DRAM / L2->SM bytes (base units) to ncu_traffic.json under
+    key CONFIG:OP:F:SCHEDULE (read by bench.py into roofline.traffic / l2_frac / dram_frac)."""
+    txt = subprocess.check_output(["ncu", "-i", path, "--page", "raw", "--csv", "--print-units", "base"]).decode()
+    rdr = list(csv.reader(io.StringIO(txt)))
+    hdr = rdr[0]
+    rows = [dict(zip(hdr, r)) for r in rdr[2:]]
+    d = max(rows, key=lambda r: float(r.get("gpu__time_duration.sum", "0").replace(",", "") or 0))
+    f = lambda k: float(d[k].replace(",", ""))
+    ent = {"dram_bytes_per_launch": f("dram__bytes_read.sum") + f("dram__bytes_write.sum"),
+           "dram_read": f("dram__bytes_read.sum"), "dram_write": f("dram__bytes_write.sum"),
+           "l2_to_sm_bytes": f("lts__t_sectors_srcunit_tex_op_read.sum") * 32,
+           "kernel_ms": f("gpu__time_duration.sum") * 1e-6,
+           "lts_throughput_pct": f("lts__throughput.avg.pct_of_peak_sustained_elapsed"),
+           "lts_hit_rate_pct": f("lts__t_sector_hit_rate.pct"),
+           "kernel": d.get("Kernel Name", "")[:100],
+           "source": f"{path} (ncu --set full --clock-control none, one launch of the bench kernel)"}
+    db = json.load(open(out)) if __import__("os").path.exists(out) else {}
+    db[key] = ent
+    json.dump(db, open(out, "w"), indent=1)
+    return ent
+
+
 if __name__ == "__main__":
     mode, path = sys.argv[1], sys.argv[2]
-    print(json.dumps(launches(path) if mode == "launches" else full(path), indent=1))
+    if mode == "traffic":
+        print(json.dumps(traffic(path, sys.argv[3]), indent=1))
+    else:
+        print(json.dumps(launches(path) if mode == "launches" else full(path), indent=1))

@@ -65,6 +65,7 @@ def candidates(cls, F, E, quick=False):
             c += [f"SV_G{g}_F{f}_P1" for g in (32, 128, 512) for f in (64, 128) if f <= max(16, 2 * F)]
         else:
             c += [f"SV_G{g}" for g in (16, 32, 64, 128, 512, 1024)]
+            c += [f"SV_G{g}_F{f}" for g in (64, 256, 512) for f in (64, 128)]     # k_dott messages + SV reduce
     else:
         c += [f"TE_G{g}_T{t}" for g in (1, 2, 4, 8) for t in Ts]
         c += [f"WE_G{g}_T1" for g in (1, 4, 16)]
@@ -73,6 +74,7 @@ def candidates(cls, F, E, quick=False):
         c += ["BV_G1_B256", "BE_G256"]
         if cls == "dot_msg":
             c += [f"SV_G{g}" for g in (16, 32, 64, 128, 512)]
+            c += [f"SV_G{g}_F{f}" for g in (64, 256, 512) for f in (64, 128)]     # k_dott (column tiles)
         else:   # message creation under SV: row chunks x column tiles, Dst_V operand hoisted
             c += [f"SV_G{g}_F{f}" for g in (16, 32, 64) for f in (16, 32, 64) if f <= max(16, F)]
     if E > 50_000_000:   # C5: drop the schedules that take seconds (atomic per-element TE at F=602)
@@ -160,6 +162,11 @@ def main():
                             results.append((ms, sched))
                     results.sort()
                     ams, _ = time_schedule(g, kw, eo, go, auto, args.reps)
+                    # the selector's own pick beside the sweep (the Fig. 12 analogue)
+                    out.write(json.dumps({"config": cfg, "class": cls, "op": nm, "F": F, "V": V, "E": E,
+                                          "mean_deg": st["mean_deg"], "cv": cv, "schedule": auto, "auto": True,
+                                          "ms": ams, "best_schedule": results[0][1], "best_ms": results[0][0],
+                                          "gbs": (by / (ams * 1e-3) / 1e9) if ams else None, "error": None}) + "\n")
                     print(f"{cfg} {cls:8s} {nm:12s} F={F:4d}  best {results[0][1]:18s} {results[0][0]:9.4f} ms  "
                           f"({by / results[0][0] / 1e6:8.1f} GB/s)  auto {auto:18s} {ams:9.4f} ms  "
                           f"worst {results[-1][1]} {results[-1][0]:.4f} ms", flush=True)

@@ -12,7 +12,7 @@ the best measured one (the Fig. 12 analogue).  Exports a plain-text tree file th
 ug_selector.cpp evaluates (selector_model.txt next to libugraph.so).
 
     python scripts/train_selector.py gpurun_out/selector_corpus.jsonl \
-        --model paper_conf_asplos_0001lslwlgslllw23_b200/selector_model.txt --report profiles/r1_selector_cv.json
+        --model paper_conf_asplos_0001lslwlgslllw23_b200/selector_model.txt --report profiles/r1/r1_selector_cv.json
 """
 import argparse
 import json

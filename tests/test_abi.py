@@ -208,6 +208,9 @@ def test_launch_counts_follow_pass2():
     assert ug.launch_count(g, "copy_lhs", "sum", schedule="TE_G4_T16", **kw) == 2
     assert ug.launch_count(g, "copy_lhs", "max", schedule="WE_G4_T1", **kw) == 3
     assert ug.launch_count(g, "copy_lhs", "mean", schedule="BV_G1", **kw) == 1
+    # SV: split rows are merged by the last-arriving chunk inside the same launch
+    assert ug.launch_count(g, "copy_lhs", "sum", schedule="SV_G2", **kw) == 1
+    assert ug.launch_count(g, "copy_lhs", "max", schedule="SV_G2_F16", **kw) == 1
     Z = torch.zeros(E, 16)
     assert ug.launch_count(g, "add", "assign", A=X, a_type="u", B=X, b_type="v", C=Z, c_type="e",
                            schedule="TE_G1_T16") == 1
