@@ -246,6 +246,38 @@ SECONDARY = [
 ]
 
 
+def headline_graph_ops(ug, torch, g, X, V, E, F, cfg, reps=5, warm=2):
+    """The other operators of the headline graph (same C5 graph and X, schedule by the selector):
+    weighted aggregation, mean / max, and the SDDMM dot (message creation and its sum) -- device
+    latency (CUDA events, median) and effective GB/s of the SURVEY 8(d) logical bytes."""
+    import ugdata
+    out = []
+    w = torch.from_numpy(ugdata.values(E, 1, cfg.seed + 1, 2, role="edge")).to(X.device)
+    cases = [("u_mul_e_sum", "mul", "sum", w, "e", "v", F), ("copy_u_mean", "copy_lhs", "mean", None, None, "v", F),
+             ("copy_u_max", "copy_lhs", "max", None, None, "v", F), ("u_dot_v", "dot", "assign", X, "v", "e", 1),
+             ("u_dot_v_sum", "dot", "sum", X, "v", "v", 1)]
+    for nm, eo, go, B, bt, ct, W in cases:
+        C = torch.empty(V if ct == "v" else E, W, device=X.device)
+        kw = dict(A=X, a_type="u", B=B, b_type=bt, C=C, c_type=ct, F=F, H=1)
+        sched = ug.schedule_select(g, eo, go, **kw)
+        ts = []
+        for i in range(warm + reps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            ug.op_run(g, eo, go, schedule=sched, **kw)
+            e1.record()
+            torch.cuda.synchronize()
+            if i >= warm:
+                ts.append(e0.elapsed_time(e1))
+        ms = statistics.median(ts)
+        by = 4 * (V + 1) + 4 * E + 4 * E * F + (4 * E if bt == "e" else (4 * V * F if bt == "v" else 0))
+        by += 4 * E * W if ct == "e" else 4 * V * W
+        out.append({"config": cfg.name if hasattr(cfg, "name") else "C5", "op": nm, "F": F, "schedule": sched,
+                    "latency_ms": round(ms, 3), "gbs": round(by / (ms * 1e-3) / 1e9, 1), "logical_bytes": by})
+        del C
+    return out
+
+
 def secondary_configs(ug, torch, dev, reps=20, warm=5):
     """Latency (median of `reps` CUDA-event timings after `warm` warm-ups) and effective GB/s,
     warm L2 (back to back) and cold L2 (a 256 MB scrub written between runs), per op x graph.
@@ -621,7 +653,9 @@ def main():
             traffic = None
 
     secondary = None
+    headline_ops = None
     if rank == 0 and world == 1 and not args.no_secondary:
+        headline_ops = headline_graph_ops(ug, torch, g, X_full[:V], V, E, F, cfg)
         secondary = secondary_configs(ug, torch, dev)
         # ncu DRAM bytes / L2 hit rate of the same (op, config, schedule), scripts/ncu_per_op.py
         pp = os.path.join(ROOT, "profiles", "ncu_per_op.json")
@@ -679,6 +713,7 @@ def main():
             "gpu_launches": launches * args.steps,
             "clocks": clocks.summary(),
             **({"dry_run": f"{backend} backend, ranks share one GPU: not a measurement"} if backend != "nccl" else {}),
+            "headline_graph_ops": headline_ops,
             "per_op_graph": secondary,
         }
         print(json.dumps(line), flush=True)

@@ -328,6 +328,12 @@ const char *ug_status_string(ug_status s);
 const char *ug_last_error(void);   /* thread-local detail of the last failing call */
 const char *ug_version(void);
 
+/* Per-call scratch (split-row partials, the pack of a misaligned A operand, k_dott partials) is
+ * allocated with cudaMallocAsync on the call's stream from the device's default memory pool --
+ * outside any framework allocator (e.g. torch's caching allocator).  The pool keeps up to 4 GiB
+ * reserved between calls; this returns everything unused to the driver (synchronises the device). */
+ug_status ug_scratch_trim(void);
+
 #ifdef __cplusplus
 }
 #endif

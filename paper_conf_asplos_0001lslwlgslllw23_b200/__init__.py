@@ -20,12 +20,17 @@ from ._ffi import (EDGE_OPS, GATHER_OPS, STRATEGIES, TTYPES, UgError, UgOpInfo, 
                    UgTensor, check, lib)
 
 __all__ = ["Graph", "op_run", "prepare", "PreparedOp", "schedule_select", "launch_count", "parse_schedule",
-           "format_schedule", "validate", "edge_permute", "selector_load", "selector_load_model", "gat_attention", "dot_attention", "op_run_arg", "arg_scatter", "reorder", "rows_gather", "Renumbered", "UgError",
+           "format_schedule", "validate", "edge_permute", "selector_load", "selector_load_model", "gat_attention", "dot_attention", "op_run_arg", "arg_scatter", "reorder", "rows_gather", "Renumbered", "UgError", "scratch_trim",
            "version"]
 
 
 def version():
     return lib.ug_version().decode()
+
+
+def scratch_trim():
+    """Return the per-call scratch the library's memory pool keeps reserved (ug_scratch_trim)."""
+    check(lib.ug_scratch_trim(), "ug_scratch_trim")
 
 
 _raw_stream = None

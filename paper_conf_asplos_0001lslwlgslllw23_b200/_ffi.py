@@ -71,6 +71,7 @@ SIGNATURES = {
     "ug_edge_permute": ([_p, _p, _p, _i32, _p], _st),
     "ug_gat_attention": ([_p, _p, _i64, _p, _i64, _p, _i64, _i32, _i32, ctypes.c_float, _p, _i64, _p, _i64, _p],
                          _st),
+    "ug_scratch_trim": ([], _st),
     "ug_dot_attention": ([_p, _p, _i64, _p, _i64, _p, _i64, _i32, _i32, _i32, ctypes.c_float, _p, _i64, _p, _i64,
                           _p], _st),
     "ug_op_run_arg": ([_p, ctypes.POINTER(UgOpInfo), _p, _i64, _p], _st),

@@ -171,6 +171,96 @@ __global__ void __launch_bounds__(256, 3) k_dotattn(GraphArgs g, DotAttnArgs a, 
     }
 }
 
+// Packed heads (Dk = Dv = D, w = D / VEC a power of two, H * w <= 32): one unit = one SV chunk
+// with ALL its heads, L = pow2(H * w) lanes, lane = h * w + i owning features h*D + i*VEC.  A
+// head's score is reduced over its w lanes by a log2(w)-step xor butterfly that leaves it in all
+// of them, so every lane runs the online softmax of its own head -- no idle lanes for small
+// heads (C2: D = 8, w = 2) and no broadcast.  UE in-edges per step.
+template <int VEC, int UE>
+__global__ void __launch_bounds__(256) k_dotattn_heads(GraphArgs g, DotAttnArgs a, const int4 *__restrict__ chunks,
+                                                       int n_chunks, int L_log2, int w_log2,
+                                                       float *__restrict__ scratch, int64_t sld) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int L = 1 << L_log2, w = 1 << w_log2;
+    const int lane = (int)(t & (L - 1));
+    const int64_t u = t >> L_log2;
+    if (u >= n_chunks) return;                    // whole units: a unit's lanes leave together
+    const int wl = threadIdx.x & 31;
+    const unsigned umask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << (wl & ~(L - 1)));
+    const int h = lane >> w_log2, i = lane & (w - 1);
+    const bool active = h < a.H;
+    const int hh = active ? h : 0;
+    const int f = hh * a.Dk + i * VEC;            // Dk == Dv
+    const int4 ch = chunks[u];
+    const int64_t v = ch.x;
+    const uint64_t keep = l2_policy_evict_last(), stream = l2_policy_evict_first();
+    float q[VEC];
+    ldg_vec<VEC>(a.q + v * a.ld_q + f, q);
+#pragma unroll
+    for (int c = 0; c < VEC; ++c) q[c] = active ? q[c] * a.scale_log2 : 0.0f;
+    const float *kb = a.k + f, *vb = a.val + f;
+    const uint32_t ldk = (uint32_t)a.ld_k, ldv = (uint32_t)a.ld_val;
+    float m = -CUDART_INF_F, den = 0.0f, acc[VEC];
+#pragma unroll
+    for (int c = 0; c < VEC; ++c) acc[c] = 0.0f;
+    const int k1 = ch.z;
+    for (int k0 = ch.y; k0 < k1; k0 += UE) {
+        const int last = k1 - 1;
+        uint32_t sidx[UE];
+#pragma unroll
+        for (int e = 0; e < UE; ++e) sidx[e] = (uint32_t)ldg_i32_hint(g.col + min(k0 + e, last), stream);
+        float kx[UE][VEC], vx[UE][VEC];
+#pragma unroll
+        for (int e = 0; e < UE; ++e) {
+            ldg_vec_hint<VEC>(kb + sidx[e] * ldk, kx[e], keep);
+            ldg_vec_hint<VEC>(vb + sidx[e] * ldv, vx[e], keep);
+        }
+        float sc[UE];
+        float mb = -CUDART_INF_F;
+#pragma unroll
+        for (int e = 0; e < UE; ++e) {
+            float p = 0.0f;
+#pragma unroll
+            for (int c = 0; c < VEC; ++c) p = __fmaf_rn(kx[e][c], q[c], p);
+            for (int off = w >> 1; off > 0; off >>= 1) p += __shfl_xor_sync(umask, p, off);
+            sc[e] = k0 + e < k1 ? p : -CUDART_INF_F;
+            if (a.attn && active && i == 0 && k0 + e < k1) {
+                const int64_t eid = g.eid ? (int64_t)g.eid[k0 + e] : (int64_t)(k0 + e);
+                a.attn[eid * a.ld_attn + h] = p;          // log2 score, normalised by k_dotattn_attn
+            }
+            mb = fmaxf(mb, sc[e]);
+        }
+        const float mn = fmaxf(m, mb);
+        const float corr = fast_exp2(m - mn);
+        den *= corr;
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) acc[c] *= corr;
+#pragma unroll
+        for (int e = 0; e < UE; ++e) {
+            const float pe = fast_exp2(sc[e] - mn);
+            den += pe;
+#pragma unroll
+            for (int c = 0; c < VEC; ++c) acc[c] = __fmaf_rn(pe, vx[e][c], acc[c]);
+        }
+        m = mn;
+    }
+    if (!active) return;
+    if (ch.w < 0) {
+        float o[VEC];
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) o[c] = den > 0.0f ? __fdiv_rn(acc[c], den) : 0.0f;
+        st_vec<VEC>(a.out + v * a.ld_out + f, o);
+        if (a.mden && i == 0) {
+            a.mden[(v * a.H + h) * 2] = m;
+            a.mden[(v * a.H + h) * 2 + 1] = den;
+        }
+    } else {
+        float *sp = scratch + ((int64_t)ch.w * a.H + h) * sld;
+        if (i == 0) { sp[0] = m; sp[1] = den; }
+        st_vec<VEC>(sp + 4 + i * VEC, acc);
+    }
+}
+
 // Split rows: merge the chunks' (max, denominator, partial sum) in chunk order.
 __global__ void k_dotattn_fix(DotAttnArgs a, const int4 *__restrict__ split, int64_t n_split,
                               const float *__restrict__ scratch, int64_t sld) {
@@ -222,11 +312,39 @@ int dotattn_vec(const DotAttnArgs &a) {
     return 0;
 }
 
+cudaError_t launch_dotattn_wide(const GraphArgs &g, const DotAttnArgs &a, int vec, int njk, int njv,
+                                const SplitPlan &plan, float *scratch, int64_t sld, cudaStream_t s);
+cudaError_t launch_dotattn_tail(const GraphArgs &g, const DotAttnArgs &a, const SplitPlan &plan, float *scratch,
+                                int64_t sld, cudaStream_t s);
+
 cudaError_t launch_dotattn(const GraphArgs &g, const DotAttnArgs &a, int vec, const SplitPlan &plan,
                            float *scratch, int64_t sld, cudaStream_t s) {
     const int njk = (int)cdiv(a.Dk, 32 * vec), njv = (int)cdiv(a.Dv, 32 * vec);
     const int64_t units = plan.n_chunks * (int64_t)a.H;
     if (units == 0) return cudaSuccess;
+    cudaError_t err = cudaSuccess;
+    const int wl = a.Dk / vec;
+    if (a.Dk == a.Dv && a.Dk % vec == 0 && (wl & (wl - 1)) == 0 && (int64_t)a.H * wl <= 32) {
+        // packed heads: one unit per chunk with all H heads (k_dotattn_heads)
+        int L = 1;
+        while (L < a.H * wl) L <<= 1;
+        const int64_t grid = cdiv(plan.n_chunks * (int64_t)L, 256);
+        const int4 *ch = reinterpret_cast<const int4 *>(plan.d_chunk);
+        UG_DISPATCH_VEC(vec, VEC,
+            k_dotattn_heads<VEC, 4><<<(unsigned)grid, 256, 0, s>>>(g, a, ch, (int)plan.n_chunks, ilog2(L),
+                                                                   ilog2(wl), scratch, sld));
+    } else {
+        err = launch_dotattn_wide(g, a, vec, njk, njv, plan, scratch, sld, s);
+    }
+    if (err == cudaSuccess) err = cudaGetLastError();
+    if (err != cudaSuccess) return err;
+    return launch_dotattn_tail(g, a, plan, scratch, sld, s);
+}
+
+// one warp per (head, chunk): heads wider than 32 lanes or not a power-of-two number of lanes
+cudaError_t launch_dotattn_wide(const GraphArgs &g, const DotAttnArgs &a, int vec, int njk, int njv,
+                                const SplitPlan &plan, float *scratch, int64_t sld, cudaStream_t s) {
+    const int64_t units = plan.n_chunks * (int64_t)a.H;
     const int64_t grid = cdiv(units, 8);
     const int4 *chunks = reinterpret_cast<const int4 *>(plan.d_chunk);
     const int nc = (int)plan.n_chunks;
@@ -253,8 +371,13 @@ cudaError_t launch_dotattn(const GraphArgs &g, const DotAttnArgs &a, int vec, co
 #undef UG_DA_K
 #undef UG_DA_V
 #undef UG_DA
-    cudaError_t err = cudaGetLastError();
-    if (err != cudaSuccess) return err;
+    return cudaGetLastError();
+}
+
+// split-row merge and optional attention normalisation (both kernel forms)
+cudaError_t launch_dotattn_tail(const GraphArgs &g, const DotAttnArgs &a, const SplitPlan &plan, float *scratch,
+                                int64_t sld, cudaStream_t s) {
+    cudaError_t err = cudaSuccess;
     if (plan.n_split_rows > 0) {
         const int64_t n = plan.n_split_rows * (int64_t)a.H * (a.Dv + 1);
         k_dotattn_fix<<<(unsigned)cdiv(n, 256), 256, 0, s>>>(a, reinterpret_cast<const int4 *>(plan.d_split),

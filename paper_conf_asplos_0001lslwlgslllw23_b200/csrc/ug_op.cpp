@@ -379,16 +379,25 @@ static int launches_for(const ug_graph *g, const Lowered &lw, const LaunchCfg &c
     return 1;
 }
 
+// Per-call scratch (split-row partials, the pack of a misaligned A, k_dott partials) comes from
+// the device's default memory pool through cudaMallocAsync on the call's stream -- outside
+// torch's caching allocator.  The pool keeps up to UG_SCRATCH_RETAIN bytes (4 GiB: the C5 pack
+// plus k_dott's partials) reserved between calls so that steady-state calls do not go back to
+// the driver; ug_scratch_trim() returns the rest.  Thread-safe (the mutex-free static init).
+#ifndef UG_SCRATCH_RETAIN
+#define UG_SCRATCH_RETAIN (4ull << 30)
+#endif
 static void ensure_pool_retains() {
-    static bool done = false;
-    if (done) return;
-    done = true;
-    int dev = 0;
-    cudaMemPool_t pool;
-    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-        uint64_t thr = UINT64_MAX;
-        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-    }
+    static const bool done = [] {
+        int dev = 0;
+        cudaMemPool_t pool;
+        if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+            uint64_t thr = UG_SCRATCH_RETAIN;
+            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+        }
+        return true;
+    }();
+    (void)done;
 }
 
 }  // namespace ug
@@ -707,7 +716,17 @@ extern "C" const char *ug_status_string(ug_status s) {
 
 extern "C" const char *ug_last_error(void) { return g_last_error.c_str(); }
 
-extern "C" const char *ug_version(void) { return "ugraph-b200 0.1 (sm_100a)"; }
+extern "C" const char *ug_version(void) { return "ugraph-b200 0.2 (sm_100a)"; }
+
+extern "C" ug_status ug_scratch_trim(void) {
+    int dev = 0;
+    cudaMemPool_t pool;
+    if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetDefaultMemPool(&pool, dev) != cudaSuccess)
+        return set_error(UG_ERR_CUDA, "ug_scratch_trim: no device pool");
+    if (cudaDeviceSynchronize() != cudaSuccess || cudaMemPoolTrimTo(pool, 0) != cudaSuccess)
+        return set_error(UG_ERR_CUDA, "ug_scratch_trim: trim failed");
+    return UG_OK;
+}
 
 // ------------------------------------------------------------------------- fused GAT chain
 namespace ug {
