@@ -4,7 +4,8 @@ out-edge operators, "transposed aggregation for grad of copy_u_sum").
 The paper is inference-only; training needs get_outedges, i.e.
 the reversed graph.  Every backward step is again a graph operator of the 160-op set:
   * d/dX of copy_u_sum(X)         = copy_u_sum over the reversed graph of dY
-  * d/dX of copy_u_mean(X)        = copy_u_sum over the reversed graph of dY / in_deg
+  * d/dX of copy_u_mean(X)        = u_div_e_sum over the reversed graph of (dY, deg_e), deg_e =
+    the in-degree of edge e's destination (one IEEE division per message, in the kernel)
   * d/dX of u_mul_e_sum(X, w)     = u_mul_e_sum over the reversed graph of (dY, w)
     (the reversed graph is built from the same COO with src / dst swapped, so edge ids -- and
     hence the rows of w -- are unchanged)
@@ -32,14 +33,16 @@ class GraphPair:
         dst = np.ascontiguousarray(dst, dtype=np.int32)
         self.fwd = Graph(self.V, src, dst)
         self.rev = Graph(self.V, dst, src)
-        self.in_deg = torch.from_numpy(np.bincount(dst, minlength=self.V).astype(np.float32))
-        self._inv_cache = {}
+        deg = np.bincount(dst, minlength=self.V).astype(np.float32)
+        self.in_deg = torch.from_numpy(deg)
+        self._deg_e_host = torch.from_numpy(deg[dst].reshape(-1, 1).copy())   # graph structure, once
+        self._deg_e = {}
 
-    def inv_in_deg(self, device):
-        if device not in self._inv_cache:
-            d = self.in_deg.to(device)
-            self._inv_cache[device] = torch.where(d > 0, 1.0 / d.clamp(min=1), torch.zeros_like(d))[:, None]
-        return self._inv_cache[device]
+    def deg_e(self, device):
+        """[E, 1]: in-degree of each edge's destination (edge-id order), the mean backward's divisor."""
+        if device not in self._deg_e:
+            self._deg_e[device] = self._deg_e_host.to(device)
+        return self._deg_e[device]
 
 
 def _agg(graph, edge_op, gather_op, X, w=None, F=None, H=1):
@@ -61,7 +64,8 @@ class _CopyUReduce(torch.autograd.Function):
         gp = ctx.gp
         g = dY.contiguous()
         if ctx.mean:
-            g = g * gp.inv_in_deg(g.device)
+            # dX[u] = sum over out-edges e = (u -> v) of dY[v] / deg(v): u_div_e_sum on the reverse
+            return None, _agg(gp.rev, "div", "sum", g, gp.deg_e(g.device)), None
         return None, _agg(gp.rev, "copy_lhs", "sum", g), None
 
 

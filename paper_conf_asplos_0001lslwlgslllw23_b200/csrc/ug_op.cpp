@@ -576,7 +576,10 @@ static ug_status run(const ug_graph *g, const ug_op_info *op, const ug_schedule 
         if (agg && plan->n_split_chunks > 0) {
             ensure_pool_retains();
             err = cudaMallocAsync((void **)&scratch, sizeof(float) * (size_t)(plan->n_split_chunks * sld), s);
-            if (err != cudaSuccess) return set_error(UG_ERR_OOM, "SV scratch allocation failed");
+            if (err != cudaSuccess) {
+                if (packed) cudaFreeAsync(packed, s);
+                return set_error(UG_ERR_OOM, "SV scratch allocation failed");
+            }
         }
         if (c.staged) {
             // B addressing mode of k_svg: none, Dst_V (any width), or a per-head / scalar Edge tensor
@@ -814,7 +817,7 @@ extern "C" ug_status ug_dot_attention(const ug_graph *g, const float *q, int64_t
     if (vec == 0) return set_error(UG_ERR_SHAPE, "ug_dot_attention: Dk and Dv must be <= 128 * vec (vec 4 / 2 / 1)");
     if ((uint64_t)g->V_total * (uint64_t)std::max(ld_k, ld_val) >= (1ull << 32))
         return set_error(UG_ERR_SHAPE, "ug_dot_attention: k / val above 2^32 elements");
-    int G = 64;
+    int G = 32;     // as the GAT traversal: split latency of the longest chunk vs merge cost
     if (const char *ev = std::getenv("UG_DOTATTN_CHUNK")) G = std::max(1, std::atoi(ev));
     const SplitPlan *plan = nullptr;
     ug_status st = get_plan(g, G, &plan);

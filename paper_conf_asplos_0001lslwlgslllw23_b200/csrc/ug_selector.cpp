@@ -53,6 +53,20 @@ struct Node {
 static std::vector<Node> g_trees[6];
 static bool g_model_loaded = false;
 
+// Learned model, nearest-neighbour form (round 2): per op class the corpus points themselves --
+// standardised, weighted features and the log-slowdown of every candidate schedule at that
+// point.  A query takes its k nearest corpus graphs, averages their log-slowdown vectors with
+// weights 1 / (distance + 1e-3), and picks the schedule with the lowest average.  Used for the
+// classes where leave-graphs-out CV favours it over the tree (scripts/train_selector.py).
+struct Knn {
+    int k = 0;
+    double w[6] = {}, mu[6] = {}, sd[6] = {};
+    std::vector<ug_schedule> scheds;
+    std::vector<std::vector<double>> X;     // [n][6] standardised * weighted
+    std::vector<std::vector<float>> Y;      // [n][n_sched] log-slowdown
+};
+static Knn g_knn[6];
+
 static int class_of(const std::string &s) {
     if (s == "msg") return 0;
     if (s == "agg") return 1;
@@ -155,10 +169,62 @@ static std::string default_model_path() {
 
 // Text format of scripts/train_selector.py: "class <name> <n>" then n lines
 // "<id> <feature> <threshold> <left> <right> <schedule|->"; '#' lines are comments.
+// Nearest-neighbour block: "knn <class> <k> <npoints> <nsched>", then lines "w ...", "mu ...",
+// "sd ..." (6 numbers each), "s <schedule> x nsched", and npoints lines "p <6 features> <nsched
+// log-slowdowns>".
+static ug_status load_knn(std::ifstream &in, std::istringstream &head, const std::string &path, Knn *out,
+                          int *cls_out) {
+    std::string name;
+    int k = 0, n = 0, ns = 0;
+    if (!(head >> name >> k >> n >> ns) || k <= 0 || n <= 0 || ns <= 0)
+        return set_error(UG_ERR_INVALID_ARG, "selector model " + path + ": bad knn header");
+    const int cls = class_of(name);
+    if (cls < 0) return set_error(UG_ERR_INVALID_ARG, "selector model: unknown class " + name);
+    Knn m;
+    m.k = k;
+    std::string line, tag;
+    for (double *arr : {m.w, m.mu, m.sd}) {
+        if (!std::getline(in, line)) return set_error(UG_ERR_INVALID_ARG, "selector model: truncated knn");
+        std::istringstream ls(line);
+        ls >> tag;
+        for (int i = 0; i < 6; ++i)
+            if (!(ls >> arr[i])) return set_error(UG_ERR_INVALID_ARG, "selector model: bad knn vector " + tag);
+    }
+    if (!std::getline(in, line)) return set_error(UG_ERR_INVALID_ARG, "selector model: truncated knn");
+    {
+        std::istringstream ls(line);
+        ls >> tag;
+        std::string sname;
+        for (int i = 0; i < ns; ++i) {
+            ug_schedule sc{};
+            if (!(ls >> sname) || ug_schedule_parse(sname.c_str(), &sc) != UG_OK)
+                return set_error(UG_ERR_INVALID_ARG, "selector model: bad knn schedule list");
+            m.scheds.push_back(sc);
+        }
+    }
+    for (int p = 0; p < n; ++p) {
+        if (!std::getline(in, line)) return set_error(UG_ERR_INVALID_ARG, "selector model: truncated knn points");
+        std::istringstream ls(line);
+        ls >> tag;
+        std::vector<double> x(6);
+        std::vector<float> y(ns);
+        for (int i = 0; i < 6; ++i)
+            if (!(ls >> x[i])) return set_error(UG_ERR_INVALID_ARG, "selector model: bad knn point");
+        for (int i = 0; i < ns; ++i)
+            if (!(ls >> y[i])) return set_error(UG_ERR_INVALID_ARG, "selector model: bad knn point");
+        m.X.push_back(std::move(x));
+        m.Y.push_back(std::move(y));
+    }
+    *out = std::move(m);
+    *cls_out = cls;
+    return UG_OK;
+}
+
 static ug_status load_model(const std::string &path, bool quiet) {
     std::ifstream in(path);
     if (!in) return quiet ? UG_OK : set_error(UG_ERR_INVALID_ARG, "cannot open " + path);
     std::vector<Node> trees[6];
+    Knn knns[6];
     std::string line;
     int cls = -1, remaining = 0;
     while (std::getline(in, line)) {
@@ -166,6 +232,15 @@ static ug_status load_model(const std::string &path, bool quiet) {
         std::istringstream ls(line);
         if (remaining == 0) {
             std::string kw, name;
+            if (line.compare(0, 4, "knn ") == 0) {
+                ls >> kw;
+                int kc = -1;
+                Knn m;
+                ug_status st = load_knn(in, ls, path, &m, &kc);
+                if (st != UG_OK) return st;
+                knns[kc] = std::move(m);
+                continue;
+            }
             int n = 0;
             if (!(ls >> kw >> name >> n) || kw != "class" || n <= 0)
                 return set_error(UG_ERR_INVALID_ARG, "selector model " + path + ": bad class line: " + line);
@@ -192,16 +267,58 @@ static ug_status load_model(const std::string &path, bool quiet) {
         --remaining;
     }
     if (remaining) return set_error(UG_ERR_INVALID_ARG, "selector model " + path + ": truncated");
-    for (int c = 0; c < 6; ++c) g_trees[c] = std::move(trees[c]);
+    for (int c = 0; c < 6; ++c) {
+        g_trees[c] = std::move(trees[c]);
+        g_knn[c] = std::move(knns[c]);
+    }
     return UG_OK;
+}
+
+static ug_schedule adapt(const Lowered &lw, ug_schedule s);
+
+// k nearest corpus graphs, distance-weighted mean log-slowdown per schedule, best first
+static std::vector<ug_schedule> knn_rank(const Knn &m, const double (&x)[6]) {
+    double z[6];
+    for (int i = 0; i < 6; ++i) z[i] = (x[i] - m.mu[i]) / m.sd[i] * m.w[i];
+    std::vector<std::pair<double, int>> d(m.X.size());
+    for (size_t p = 0; p < m.X.size(); ++p) {
+        double s = 0;
+        for (int i = 0; i < 6; ++i) s += (z[i] - m.X[p][i]) * (z[i] - m.X[p][i]);
+        d[p] = {std::sqrt(s), (int)p};
+    }
+    const size_t k = std::min<size_t>((size_t)m.k, d.size());
+    std::partial_sort(d.begin(), d.begin() + k, d.end());
+    std::vector<std::pair<double, int>> score(m.scheds.size());
+    for (size_t j = 0; j < m.scheds.size(); ++j) score[j] = {0.0, (int)j};
+    double wsum = 0;
+    for (size_t q = 0; q < k; ++q) {
+        const double wt = 1.0 / (d[q].first + 1e-3);
+        wsum += wt;
+        for (size_t j = 0; j < m.scheds.size(); ++j) score[j].first += wt * m.Y[d[q].second][j];
+    }
+    std::sort(score.begin(), score.end());
+    std::vector<ug_schedule> out;
+    for (auto &sc : score) out.push_back(m.scheds[sc.second]);
+    (void)wsum;
+    return out;
 }
 
 static bool model_select(const ug_graph *g, const Lowered &lw, ug_schedule *out) {
     const std::vector<Node> &t = g_trees[lw.op_class];
-    if (t.empty() || g->V <= 0 || g->E <= 0) return false;
+    const Knn &m = g_knn[lw.op_class];
+    if ((t.empty() && m.k == 0) || g->V <= 0 || g->E <= 0) return false;
     const double mean = std::max(g->mean_deg, 1e-9);
     const double x[6] = {std::log2((double)g->V), std::log2((double)g->E), std::log2(mean), g->std_nnz / mean,
                          std::log2(std::max<double>(1.0, (double)g->max_deg) / mean), std::log2((double)lw.args.F)};
+    if (m.k > 0) {
+        // the best-ranked schedule that resolves on this operator's layout
+        for (const ug_schedule &sc : knn_rank(m, x)) {
+            ug_schedule s2 = adapt(lw, sc);
+            LaunchCfg cfg;
+            if (resolve(g, lw, s2, &cfg) == UG_OK) { *out = s2; return true; }
+        }
+        return false;
+    }
     int n = 0;
     for (int steps = 0; steps < 64 && t[n].feature >= 0; ++steps) n = x[t[n].feature] <= t[n].thr ? t[n].left : t[n].right;
     if (t[n].feature >= 0) return false;
@@ -233,13 +350,20 @@ static ug_schedule prior(const ug_graph *g, const Lowered &lw) {
     while (lanes < chunks && lanes < 32) lanes <<= 1;
     if (lw.op_class == 0) {            // message creation: thread-edge (Table 9: always TE)
         s.strategy = UG_TE; s.group = 1; s.tile = lanes;
-    } else if (lw.op_class == 2) {     // SDDMM: lanes over the head's D features
-        int dl = 1;
-        const int dch = (lw.args.D + vec - 1) / vec;
-        while (dl < dch && dl < 32) dl <<= 1;
-        s.strategy = UG_TE; s.group = 1; s.tile = dl;
-    } else if (lw.op_class == 3) {
-        s.strategy = UG_WV; s.group = 1; s.tile = 1;
+    } else if (lw.op_class == 2 || lw.op_class == 3) {
+        const Operand &A = lw.args.A, &B = lw.args.B;
+        const bool uv = A.div == 1 && B.div == 1 &&
+                        ((A.type == UG_T_SRC_V && B.type == UG_T_DST_V) || (A.type == UG_T_DST_V && B.type == UG_T_SRC_V));
+        if (uv && lw.args.D >= 256) {                 // wide heads: column-tiled k_dott (r2 sweep, C5)
+            s.strategy = UG_SV; s.group = 512; s.ftile = 128;
+        } else if (lw.op_class == 2) {                // SDDMM: lanes over the head's D features
+            int dl = 1;
+            const int dch = (lw.args.D + vec - 1) / vec;
+            while (dl < dch && dl < 32) dl <<= 1;
+            s.strategy = UG_TE; s.group = 1; s.tile = dl;
+        } else {
+            s.strategy = UG_WV; s.group = 1; s.tile = 1;
+        }
     } else {                           // aggregation (classes 1, 4, 5)
         if (W >= 32 || g->max_deg > 256) {
             s.strategy = UG_SV; s.group = 512; s.ftile = 0;

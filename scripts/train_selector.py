@@ -82,6 +82,51 @@ def cv_eval(X, Y, T, groups, depth, leaf, folds=6):
     return np.array(slow)
 
 
+def knn_scores(Xtr, Ytr, Xte, k, w):
+    """Distance-weighted mean log-slowdown of the k nearest training points (standardised,
+    weighted features) -- the rule ug_selector.cpp's knn_rank evaluates."""
+    mu, sd = Xtr.mean(axis=0), Xtr.std(axis=0) + 1e-9
+    Ztr, Zte = (Xtr - mu) / sd * w, (Xte - mu) / sd * w
+    out = np.empty((len(Xte), Ytr.shape[1]))
+    for i, z in enumerate(Zte):
+        d = np.sqrt(((Ztr - z) ** 2).sum(axis=1))
+        nn = np.argsort(d, kind="stable")[:k]
+        wt = 1.0 / (d[nn] + 1e-3)
+        out[i] = (Ytr[nn] * wt[:, None]).sum(axis=0) / wt.sum()
+    return out
+
+
+def knn_cv_eval(X, Y, T, groups, k, w, folds=6):
+    """Leave-graphs-out CV of the nearest-neighbour rule (same folds as cv_eval)."""
+    ug = np.unique(groups)
+    rng = np.random.default_rng(0)
+    rng.shuffle(ug)
+    slow = []
+    for f in range(folds):
+        test_g = set(ug[f::folds].tolist())
+        te = np.array([g in test_g for g in groups])
+        if te.all() or not te.any():
+            continue
+        pred = knn_scores(X[~te], Y[~te], X[te], k, w).argmin(axis=1)
+        tt = T[te]
+        best = tt.min(axis=1)
+        chosen = tt[np.arange(len(pred)), pred]
+        chosen = np.where(np.isfinite(chosen), chosen, best * 20.0)
+        slow += (chosen / best).tolist()
+    return np.array(slow)
+
+
+def export_knn(X, Y, scheds, cls, k, w):
+    mu, sd = X.mean(axis=0), X.std(axis=0) + 1e-9
+    Z = (X - mu) / sd * w
+    lines = [f"knn {cls} {k} {len(X)} {len(scheds)}",
+             "w " + " ".join(f"{v:.9g}" for v in w), "mu " + " ".join(f"{v:.9g}" for v in mu),
+             "sd " + " ".join(f"{v:.9g}" for v in sd), "s " + " ".join(scheds)]
+    for z, y in zip(Z, Y):
+        lines.append("p " + " ".join(f"{v:.6g}" for v in z) + " " + " ".join(f"{v:.5g}" for v in y))
+    return lines
+
+
 def export_tree(model, scheds, cls):
     t = model.tree_
     lines = [f"class {cls} {t.node_count}"]
@@ -116,9 +161,11 @@ def main():
     ap.add_argument("--leaf", type=int, default=3)
     args = ap.parse_args()
     rows = load(args.corpus)
-    out = ["# ugraph-b200 learned selector v1 (scripts/train_selector.py): per op class a regression",
+    out = ["# ugraph-b200 learned selector v2 (scripts/train_selector.py): per op class either a regression",
            "# tree over " + " ".join(FEATURES) + "; node: id feature threshold left right schedule",
-           "# (x[feature] <= threshold -> left; leaves have feature -1 and name their schedule)"]
+           "# (x[feature] <= threshold -> left; leaves have feature -1 and name their schedule), or a",
+           "# nearest-neighbour block (knn <class> <k> <n> <nsched>; w / mu / sd; s <schedules>; p <z> <log-slowdowns>)",
+           "# -- whichever leave-graphs-out CV favours"]
     report = {"features": FEATURES, "classes": {}}
     for cls in sorted({r["class"] for r in rows}):
         rc = [r for r in rows if r["class"] == cls]
@@ -132,17 +179,35 @@ def main():
             res[d] = {"geomean": float(np.exp(np.log(s).mean())), "p90": float(np.quantile(s, 0.9)),
                       "max": float(s.max()), "within_10pct": float((s <= 1.10).mean())}
         d_best = min(res, key=lambda d: res[d]["geomean"])
-        model = fit(X, Y, d_best, args.leaf)
-        out += export_tree(model, scheds, cls)
+        # the nearest-neighbour rule over the same folds; the better of the two is exported
+        kres = {}
+        for k in (3, 5, 8):
+            for fw in (1.0, 2.0, 4.0):
+                w = np.array([1.0, 1.0, 1.0, 1.0, 1.0, fw])
+                sk = knn_cv_eval(X, Y, T, groups, k, w)
+                kres[f"k{k}_wF{fw:g}"] = {"k": k, "wF": fw, "geomean": float(np.exp(np.log(sk).mean())),
+                                          "p90": float(np.quantile(sk, 0.9)), "max": float(sk.max()),
+                                          "within_10pct": float((sk <= 1.10).mean())}
+        kb = min(kres, key=lambda key: kres[key]["geomean"])
+        use_knn = kres[kb]["geomean"] < res[d_best]["geomean"]
+        if use_knn:
+            w = np.array([1.0, 1.0, 1.0, 1.0, 1.0, kres[kb]["wF"]])
+            out += export_knn(X, Y, scheds, cls, kres[kb]["k"], w)
+        else:
+            model = fit(X, Y, d_best, args.leaf)
+            out += export_tree(model, scheds, cls)
         report["classes"][cls] = {"points": len(rc), "graphs": int(len(np.unique(groups))),
                                   "schedules": len(scheds), "depth": d_best, "cv_by_depth": res,
+                                  "knn_cv": kres, "knn_best": kb, "exported": "knn" if use_knn else "tree",
                                   "fixed_best": {"schedule": scheds[best_fixed],
                                                  "geomean": float(np.exp(np.log(fixed).mean())),
                                                  "p90": float(np.quantile(fixed, 0.9))}}
-        print(f"{cls:8s} points {len(rc):4d}  depth {d_best}  CV geomean slowdown "
+        print(f"{cls:8s} points {len(rc):4d}  tree depth {d_best}: CV geomean slowdown "
               f"{res[d_best]['geomean']:.3f} p90 {res[d_best]['p90']:.3f} within10% "
-              f"{res[d_best]['within_10pct']:.2f} | single best schedule {scheds[best_fixed]} geomean "
-              f"{report['classes'][cls]['fixed_best']['geomean']:.3f}", flush=True)
+              f"{res[d_best]['within_10pct']:.2f} | knn {kb}: {kres[kb]['geomean']:.3f} p90 {kres[kb]['p90']:.3f} "
+              f"within10% {kres[kb]['within_10pct']:.2f} -> {'knn' if use_knn else 'tree'} | single best "
+              f"schedule {scheds[best_fixed]} geomean {report['classes'][cls]['fixed_best']['geomean']:.3f}",
+              flush=True)
     with open(args.model, "w") as f:
         f.write("\n".join(out) + "\n")
     if args.report:

@@ -1,10 +1,17 @@
-"""Backward through the unified operator vs torch autograd of a float64
-index_add_ reference on the same graph."""
+"""Backward through the unified operator.
+
+Two checks per operator: (1) parity -- the forward and every gradient against the ORACLE
+evaluating the backward's defining graph operator (the transposed aggregation over the reversed
+graph, u_div_e_sum for the mean, u_dot_v for the edge-weight gradient) within 1e-5 * sum|terms|
+(R11); (2) calculus -- the same gradients against torch autograd of a float64 index_add_
+reference, which shows those operators ARE the gradients."""
 import numpy as np
 import pytest
 import torch
 
+import oracle
 import ugdata
+from gpu_util import assert_parity
 
 pytestmark = pytest.mark.gpu
 
@@ -38,6 +45,12 @@ def ref_agg(V, src, dst, X, w=None, mean=False):
     return Y
 
 
+def oracle_check(got, op, V, src, dst, A, a_type, B=None, b_type=None, c_type="v", F=None, H=1, what=""):
+    ref, bnd = oracle.op(V, src, dst, op[0], op[1], A=A, a_type=a_type, B=B, b_type=b_type, c_type=c_type,
+                         F=F or A.shape[1], H=H, bound=True)
+    assert_parity((op[0], a_type, b_type, op[1], c_type), got.detach().cpu().numpy(), ref, bnd, False, what=what)
+
+
 def check(a, b, rtol=1e-5):
     b = b.float()
     torch.testing.assert_close(a, b, rtol=rtol, atol=rtol * (b.abs().max().item() + 1e-6))
@@ -55,6 +68,13 @@ def test_copy_u_sum_mean_backward(graph, mean):
     (Yr * G.double()).sum().backward()
     check(Y.detach(), Yr.detach())
     check(X.grad, X64.grad)
+    Xn, Gn = X.detach().cpu().numpy(), G.cpu().numpy()
+    oracle_check(Y, ("copy_lhs", "mean" if mean else "sum"), V, src, dst, Xn, "u", what="forward")
+    if mean:
+        deg_e = np.bincount(dst, minlength=V).astype(np.float32)[dst].reshape(-1, 1)
+        oracle_check(X.grad, ("div", "sum"), V, dst, src, Gn, "u", deg_e, "e", what="mean backward")
+    else:
+        oracle_check(X.grad, ("copy_lhs", "sum"), V, dst, src, Gn, "u", what="sum backward")
 
 
 @pytest.mark.parametrize("H", [1, 4])
@@ -73,3 +93,7 @@ def test_u_mul_e_sum_backward(graph, H):
     check(Y.detach(), Yr.detach())
     check(X.grad, X64.grad)
     check(w.grad, w64.grad)
+    Xn, Gn, wn = X.detach().cpu().numpy(), G.cpu().numpy(), w.detach().cpu().numpy()
+    oracle_check(Y, ("mul", "sum"), V, src, dst, Xn, "u", wn, "e", H=H, what="forward")
+    oracle_check(X.grad, ("mul", "sum"), V, dst, src, Gn, "u", wn, "e", H=H, what="dX")
+    oracle_check(w.grad, ("dot", "assign"), V, src, dst, Xn, "u", Gn, "v", c_type="e", F=32, H=H, what="dw")

@@ -86,9 +86,41 @@ def test_shipped_model_parses():
     if not os.path.exists(path):
         pytest.skip("no trained model shipped")
     ug.selector_load_model(path)
+    in_knn = 0
     for ln in open(path):
         if ln.startswith("#") or ln.startswith("class"):
             continue
         parts = ln.split()
+        if parts[0] == "knn":
+            in_knn = 1
+            continue
+        if parts[0] in ("w", "mu", "sd", "p"):
+            continue
+        if parts[0] == "s":
+            for sc in parts[1:]:
+                ug.parse_schedule(sc)
+            continue
         if parts[1] == "-1":
             ug.parse_schedule(parts[5])
+
+
+@pytest.mark.parametrize("sigma", [0.3, 1.4])
+@pytest.mark.parametrize("F", [16, 128])
+def test_knn_matches_reference(empty_table, sigma, F):
+    """The C++ nearest-neighbour rule picks the schedule train_selector.knn_scores ranks first."""
+    rng = np.random.default_rng(3)
+    X = np.column_stack([rng.uniform(11, 18, 40), rng.uniform(14, 23, 40), rng.uniform(1, 6, 40),
+                         rng.uniform(0.3, 2.0, 40), rng.uniform(1, 8, 40), rng.choice([3, 4, 5, 6, 7], 40)])
+    scheds = ["TE_G8_T4", "WE_G4_T1", "SV_G32_F32", "WV_G1_T1"]
+    Y = rng.uniform(0, 1.5, (40, len(scheds)))
+    w = np.array([1, 1, 1, 1, 1, 2.0])
+    p = empty_table / "knn.txt"
+    p.write_text("\n".join(train_selector.export_knn(X, Y, scheds, "agg", 5, w)) + "\n")
+    ug.selector_load_model(str(p))
+    V = 3000
+    src, dst = ugdata.chung_lu(V, 30000, True, sigma, 0.5, 5)
+    g = ug.Graph(V, src, dst, host_only=True)
+    x = np.array([_features(g.stats(), F)])
+    want = scheds[int(train_selector.knn_scores(X, Y, x, 5, w)[0].argmin())]
+    got = _select(g, V, F)
+    assert got.split("_")[0] == want.split("_")[0] and got.split("_")[1] == want.split("_")[1], (got, want)
