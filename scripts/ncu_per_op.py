@@ -60,8 +60,8 @@ def parse(csv_path, order_path, out_path):
         d = launches.setdefault(int(r["ID"]), {"kernel": r["Kernel Name"].split("(")[0]})
         unit = r.get("Metric Unit", "")
         v = float(r["Metric Value"].replace(",", ""))
-        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-3, "usecond": 1.0,
-                 "msecond": 1e3, "sector": 1, "%": 1}.get(unit, 1)
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1e-3, "nsecond": 1e-3, "us": 1.0,
+                 "usecond": 1.0, "ms": 1e3, "msecond": 1e3, "sector": 1, "%": 1}.get(unit, 1)   # time -> us
         d[r["Metric Name"]] = v * scale
     seq = [launches[k] for k in sorted(launches)]
     order = json.load(open(order_path))
