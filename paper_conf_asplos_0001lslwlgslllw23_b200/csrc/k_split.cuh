@@ -54,6 +54,24 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
         float m[UF][VEC];
 #pragma unroll
         for (int q = 0; q < UF; ++q) ldg_vec_hint<VEC>(Ab + (s[q] * lda + fo), m[q], keep);
+#ifndef UG_MUL_FMA
+#define UG_MUL_FMA 0
+#endif
+        // UG_MUL_FMA: a per-edge scalar weight folded into the sum by FMA (the message is then not
+        // rounded on its own -- within R11's bound, exact in integer mode); A/B switch
+        constexpr bool FMA_W = UG_MUL_FMA && BM == 2 && KE == K_MUL && (GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN);
+        if constexpr (FMA_W) {
+            float wq[UF];
+#pragma unroll
+            for (int q = 0; q < UF; ++q) wq[q] = __ldg(op.B.p + ((uint32_t)(PRED ? min(k + q, kl) : k + q) * ldb + cbo));
+#pragma unroll
+            for (int q = 0; q < UF; ++q) {
+                const bool ok = !PRED || k + q < k1;
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) acc[i] = ok ? __fmaf_rn(m[q][i], wq[q], acc[i]) : acc[i];
+            }
+            return;
+        }
         if constexpr (BM != 0) {
 #pragma unroll
             for (int q = 0; q < UF; ++q) {

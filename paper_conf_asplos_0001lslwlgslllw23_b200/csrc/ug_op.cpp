@@ -108,7 +108,7 @@ ug_status lower(const ug_graph *g, const ug_op_info *op, Lowered *out) {
         for (int v : {4, 2}) {
             const bool ok = o.div == 1 ? (o.ld % v == 0) && ((uintptr_t)o.p % (4 * v) == 0) &&
                                              (span % v == 0 || o.ld >= ((F + v - 1) / v) * v)
-                                       : (o.div % v == 0);
+                                       : (o.div % v == 0 || o.div == F);   // a scalar (width 1) broadcasts over every chunk
             if (ok) return v;
         }
         return 1;
