@@ -449,6 +449,7 @@ extern "C" ug_status ug_selector_load_model(const char *path) {
     ug::g_model_loaded = true;
     if (!*path) {                       // "" unloads the model
         for (auto &t : ug::g_trees) t.clear();
+        for (auto &m : ug::g_knn) m = ug::Knn{};
         return UG_OK;
     }
     return ug::load_model(path, false);
