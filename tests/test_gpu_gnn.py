@@ -135,3 +135,22 @@ def test_gat_layer(c2, fused):
     deg = np.bincount(dst, minlength=V).astype(np.float64)[:, None]
     tol = 1e-5 * bnd if fused else 1e-5 * bnd + (deg + 8) * U * bnd
     within(out, ref, tol, f"GAT fused={fused}")
+
+
+@pytest.mark.parametrize("fused", [True, False])
+def test_dotgat_layer(c2, fused):
+    """Dot-product attention layer: the fused ug_dot_attention traversal and the unfused operator
+    chain, both against oracle.dot_attention on the layer's own z (R25 bound; the unfused chain
+    adds the rounding of its separately stored scores, exp and denominator, as in test_gat_layer)."""
+    V, src, dst, gd = c2
+    torch.manual_seed(3)
+    H, D = 4, 16
+    layer = gnn.DotGATConv(16, D, H).cuda()
+    h = torch.randn(V, 16, device="cuda")
+    with torch.no_grad():
+        out = layer(gd, h, fused=fused)
+        z = (h @ layer.W).cpu().numpy()
+    ref, attn, bnd = oracle.dot_attention(V, src, dst, z, z, z, H, scale=1.0 / D ** 0.5, bound=True)
+    deg = np.bincount(dst, minlength=V).astype(np.float64)[:, None]
+    tol = 1e-5 * bnd if fused else 1e-5 * bnd + (deg + 16) * U * bnd
+    within(out, ref, tol, f"DotGAT fused={fused}")
