@@ -343,6 +343,35 @@ def secondary_configs(ug, torch, dev, reps=20, warm=5):
         del A, B, C
     del scrub
     out.append(gat_chain_graph(ug, torch, dev, graphs["C2"][0]))
+    out += dot_attention_graphs(ug, torch, dev, graphs)
+    return out
+
+
+def dot_attention_graphs(ug, torch, dev, graphs, reps=20):
+    """Fused dot-product attention (ug_dot_attention, f3) on the C2 / C4 shapes: device latency
+    (queued behind a spin kernel) and effective GB/s of its logical bytes (row_ptr, col_idx, the
+    q row per destination, the k and val rows per edge, the output)."""
+    import ugdata
+    out = []
+    for cfg, H, F in (("C2", 8, 64), ("C4", 8, 128), ("C4", 1, 128)):
+        g, E = graphs[cfg]
+        V = ugdata.CONFIGS[cfg].V
+        z = torch.randn(V, F, device=dev)
+        o = torch.empty(V, F, device=dev)
+        ts = []
+        for i in range(5 + reps):
+            torch.cuda._sleep(200_000)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            ug.dot_attention(g, z, z, z, H, out=o)
+            e1.record()
+            torch.cuda.synchronize()
+            if i >= 5:
+                ts.append(e0.elapsed_time(e1) * 1e3)
+        us = statistics.median(ts)
+        by = 4 * (V + 1) + 4 * E + 4 * V * F + 2 * 4 * E * F + 4 * V * F
+        out.append({"config": cfg, "op": "dot attention (fused SDDMM + softmax + SpMM)", "F": F, "H": H,
+                    "latency_us": round(us, 2), "logical_bytes": by, "gbs": round(by / (us * 1e-6) / 1e9, 1)})
     return out
 
 

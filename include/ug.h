@@ -20,7 +20,16 @@
  *   - The library never keeps a caller pointer after a call returns (graphs copy their
  *     input).  The caller owns A, B, C.
  *   - ug_op_run is asynchronous (no host synchronisation) and re-entrant across streams;
- *     graphs are immutable after creation.
+ *     graphs are immutable after creation.  Per-call scratch is stream-ordered
+ *     (cudaMallocAsync on the call's stream).  The single-launch merges of split rows
+ *     (ug_op_run under SV for small operators, ug_gat_attention, ug_op_run_arg) count chunk
+ *     arrivals in a per-(graph, stream) counter buffer that every call leaves zeroed: calls on
+ *     different streams never share one.  Restriction: a CUDA graph captured on stream S
+ *     embeds S's counters, so two replays of it -- or a replay and an eager call on S -- must
+ *     not run concurrently.
+ *   - The first call of a graph with a given SV chunk size builds and uploads its plan (and
+ *     counters) synchronously, in relaxed stream-capture mode: that first call may itself be
+ *     inside a CUDA-graph capture.
  */
 #ifndef UG_H_
 #define UG_H_
@@ -266,8 +275,8 @@ ug_status ug_edge_permute(const ug_graph *g, const float *in, float *out, int32_
  *   out [V][F] (ld_out): device fp32, every row written; zero in-degree rows -> 0 (R7).
  *   attn: NULL, or device fp32 [E][H] (ld_attn) receiving a(e,h) at row = edge id (R9).
  *   Accuracy: within 1e-5 * sum_e a(e,h) |z[u][f]| of the fp64 definition (oracle.gat);
- *   attention within 1e-5 relative.  Deterministic (no atomics).  One kernel launch on
- *   `stream`; the first call per graph uploads a small row list synchronously.
+ *   attention within 1e-5 relative.  Deterministic (chunk-order merge).  One kernel launch on
+ *   `stream` (re-entrancy and capture: see the conventions at the top).
  *   Errors: UG_ERR_INVALID_ARG (NULL graph / data, host-only graph), UG_ERR_SHAPE (H <= 0,
  *   H does not divide F, ld < width), UG_ERR_OOM, UG_ERR_CUDA.
  */
