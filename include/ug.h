@@ -116,7 +116,7 @@ typedef struct {
     int32_t block_threads;  /* CTA size (0 -> 256)                                              */
     int32_t ftile;          /* column-tile width for L2 blocking, tile-major grid order; 0 = off */
     int32_t vec;            /* feature vector width 1/2/4; 0 -> widest the layout allows        */
-    int32_t flags;          /* UG_SCHED_PACK | UG_SCHED_TMA | UG_SCHED_ASYNC.  UG_SCHED_PACK (SV only): first stage a full-width Src_V operand whose
+    int32_t flags;          /* UG_SCHED_PACK | UG_SCHED_TMA | UG_SCHED_ASYNC | UG_SCHED_EDGELANES.  UG_SCHED_PACK (SV only): first stage a full-width Src_V operand whose
                                rows are not 128-byte aligned into an aligned scratch copy, so each
                                column slab occupies whole L2 lines and rows take 16-byte loads   */
 } ug_schedule;
@@ -126,6 +126,11 @@ typedef struct {
                              by TMA (cp.async.bulk.tensor tile::gather4, issued by one lane per
                              warp) into a per-warp ring of shared-memory stages completed on
                              mbarriers, instead of into registers                                */
+#define UG_SCHED_EDGELANES 8  /* WV aggregation with W / vec <= 8 ("_E1"): the 32 lanes of a warp take
+                                 a destination row's in-edges round-robin and reduce all its
+                                 features in registers, then combine by an xor butterfly -- one
+                                 launch, owner computes; for narrow features on small, skewed
+                                 graphs, where feature lanes leave most lanes idle             */
 #define UG_SCHED_ASYNC 4  /* SV aggregation only ("_A1"): the same ring filled by cp.async
                              (LDGSTS, each lane its own features of the group's four rows).
                              Both staged forms: ftile = 32 * vec columns (128 / 64 / 32), a

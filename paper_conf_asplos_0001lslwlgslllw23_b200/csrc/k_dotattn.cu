@@ -14,6 +14,8 @@
 // (max, denominator, partial sum) per chunk and k_dotattn_fix merges them in chunk order
 // (deterministic).  With attn requested, the raw log2 scores are stored during the traversal and
 // k_dotattn_attn normalises them with each row's final (max, denominator).
+#include <cstdlib>
+
 #include "k_split.cuh"
 
 namespace ug {
@@ -324,7 +326,12 @@ cudaError_t launch_dotattn(const GraphArgs &g, const DotAttnArgs &a, int vec, co
     if (units == 0) return cudaSuccess;
     cudaError_t err = cudaSuccess;
     const int wl = a.Dk / vec;
-    if (a.Dk == a.Dv && a.Dk % vec == 0 && (wl & (wl - 1)) == 0 && (int64_t)a.H * wl <= 32) {
+    static const bool force_wide = std::getenv("UG_DOTATTN_WIDE") != nullptr;   // A/B switch
+    // packed heads when a head spans <= 8 lanes (<= 3 butterfly steps per edge); wider heads reduce
+    // 8 edges at once by the transposed butterfly (C4 H = 1, D = 128: 303 -> 226 us; H = 8: packed
+    // 236 us vs 1,288 us; profiles/r2/ab_r2t.log)
+    if (!force_wide && a.Dk == a.Dv && a.Dk % vec == 0 && (wl & (wl - 1)) == 0 && wl <= 8 &&
+        (int64_t)a.H * wl <= 32) {
         // packed heads: one unit per chunk with all H heads (k_dotattn_heads)
         int L = 1;
         while (L < a.H * wl) L <<= 1;

@@ -85,7 +85,12 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
                     if constexpr (bfull) {
                         ldg_vec_hint<VEC>(bp, b, BM == 3 ? stream : keep);
                     } else {
+#ifdef UG_EXPERIMENT_NO_WEIGHT_LOAD
+                        // timing experiment only (wrong results): the per-edge weight load removed
+                        const float x = 1.0f + (float)(row & 1) * (float)(uintptr_t)bp * 0.0f;
+#else
                         const float x = __ldg(bp);
+#endif
 #pragma unroll
                         for (int i = 0; i < VEC; ++i) b[i] = x;
                     }

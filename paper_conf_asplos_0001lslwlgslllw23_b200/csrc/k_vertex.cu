@@ -98,4 +98,87 @@ cudaError_t launch_vertex(int kedge, int gather, const GraphArgs &g, const OpArg
     return cudaGetLastError();
 }
 
+// Edge-lanes warp-vertex ("WV_..._E1", round 2): for narrow features (W / VEC <= 8 chunks) the
+// lanes of a warp split a destination row's IN-EDGES instead of its features -- lane l takes
+// edges k0 + l, k0 + l + 32, ... and reduces every feature of its messages in registers, then an
+// xor butterfly over the 32 lanes combines them (owner computes: one launch, no atomics, no
+// init).  A row of in-degree d costs ceil(d / 32) dependent gather steps instead of d / UF, which
+// is what bounds small, skewed graphs (C1 / C2) under the feature-lane schedules.
+template <int KE, int GOP, int VEC, int NC>
+__global__ void __launch_bounds__(256) k_vertex_el(GraphArgs g, OpArgs op, int G) {
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    const int64_t v0 = warp * G;
+    if (v0 >= g.V) return;                            // whole warps leave together
+    const int64_t v_end = min(g.V, v0 + (int64_t)G);
+    int64_t ca[NC], cb[NC];
+#pragma unroll
+    for (int j = 0; j < NC; ++j) {
+        ca[j] = op_col(op.A, min(j * VEC, op.W - 1));
+        cb[j] = op_col(op.B, min(j * VEC, op.W - 1));
+    }
+    for (int64_t v = v0; v < v_end; ++v) {
+        const int64_t k0 = (int64_t)g.row_ptr[v] - g.rp_base;
+        const int64_t k1 = (int64_t)g.row_ptr[v + 1] - g.rp_base;
+        float acc[NC][VEC];
+#pragma unroll
+        for (int j = 0; j < NC; ++j)
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) acc[j][i] = g_init<GOP>();
+        for (int64_t k = k0 + lane; k < k1; k += 32) {
+            const int64_t src = g.col[k];
+            const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
+            const int64_t ra = op_row(op.A.type, src, v, e);
+            const int64_t rb = op_row(op.B.type, src, v, e);
+#pragma unroll
+            for (int j = 0; j < NC; ++j) {
+                if (j * VEC < op.W) {
+                    float m[VEC];
+                    message<KE, VEC>(op, ra, ca[j], rb, cb[j], m);
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i) acc[j][i] = g_combine<GOP>(acc[j][i], m[i]);
+                }
+            }
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1)
+#pragma unroll
+            for (int j = 0; j < NC; ++j)
+#pragma unroll
+                for (int i = 0; i < VEC; ++i)
+                    acc[j][i] = g_combine<GOP>(acc[j][i], __shfl_xor_sync(0xffffffffu, acc[j][i], off));
+        const int64_t deg = k1 - k0;
+#pragma unroll
+        for (int j = 0; j < NC; ++j) {
+            if (lane == j && j * VEC < op.W) {        // lane j stores chunk j
+                float o[VEC];
+#pragma unroll
+                for (int i = 0; i < VEC; ++i) o[i] = g_finalize<GOP>(acc[j][i], deg);
+                st_out<VEC>(op.C + v * op.c_ld + j * VEC, o, op.W - j * VEC, op.c_vec);
+            }
+        }
+    }
+}
+
+cudaError_t launch_vertex_el(int kedge, int gather, const GraphArgs &g, const OpArgs &op, const LaunchCfg &c,
+                             cudaStream_t s) {
+    const int nc = (int)cdiv(op.W, c.vec);
+    const int64_t warps = cdiv(g.V, c.G);
+    if (warps == 0) return cudaSuccess;
+    const int64_t grid = cdiv(warps * 32, 256);
+#define UG_EL(NCV)                                                                                       \
+    UG_DISPATCH_KE(kedge, KE,                                                                            \
+        UG_DISPATCH_RED(gather, GOP, k_vertex_el<KE, GOP, VEC, NCV><<<(unsigned)grid, 256, 0, s>>>(g, op, c.G)))
+    UG_DISPATCH_VEC(c.vec, VEC, {
+        switch (nc) {
+        case 1: UG_EL(1); break;
+        case 2: UG_EL(2); break;
+        case 3: case 4: UG_EL(4); break;
+        default: UG_EL(8); break;
+        }
+    });
+#undef UG_EL
+    return cudaGetLastError();
+}
+
 }  // namespace ug

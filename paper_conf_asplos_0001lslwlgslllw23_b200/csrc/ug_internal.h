@@ -56,6 +56,7 @@ struct LaunchCfg {
     int ftile;        // column tile width (multiple of vec), 0 = whole width
     int vec;          // 1, 2, 4
     bool pack;        // UG_SCHED_PACK: stage A into 128-byte-aligned rows first (SV only)
+    bool edgelanes;   // WV aggregation with lanes over a row's in-edges (k_vertex_el)
     bool dott;        // SV dot with column tiles (k_dott): any head width, tile-major partials
     int staged;       // SV aggregation with shared-memory row staging (k_svg): 0 off,
                       // 1 UG_SCHED_TMA (TMA gather4), 2 UG_SCHED_ASYNC (cp.async / LDGSTS)
@@ -74,6 +75,8 @@ struct SplitPlan {
 // Kernel launchers (kernels/*.cu).  All return cudaGetLastError().
 cudaError_t launch_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
                           const LaunchCfg &c, cudaStream_t s);
+cudaError_t launch_vertex_el(int kedge, int gather, const GraphArgs &g, const OpArgs &op, const LaunchCfg &c,
+                             cudaStream_t s);
 cudaError_t launch_edge(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
                         const LaunchCfg &c, cudaStream_t s);
 cudaError_t launch_block_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,

@@ -153,6 +153,21 @@ ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, La
     // SV stores through any C alignment (st_out), so its vector width is bounded by the operands
     // only; with UG_SCHED_PACK the staged copy of A is 16-byte aligned (a_vec = 4).
     c.pack = c.strategy == UG_SV && (s.flags & UG_SCHED_PACK) && lw.pack_ok;
+    if (s.flags & UG_SCHED_EDGELANES) {
+        // lanes over a row's in-edges (k_vertex_el): WV aggregation of an elementwise message, narrow W
+        if (c.strategy != UG_WV || lw.dot || lw.to_edges)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "_E1: WV aggregation of an elementwise message only");
+        c.vec = s.vec ? s.vec : lw.max_vec;
+        if (c.vec > lw.max_vec) return set_error(UG_ERR_ALIGNMENT, "forced vec wider than the operand layout allows");
+        if ((lw.args.W + c.vec - 1) / c.vec > 8)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "_E1: at most 8 feature vectors per row (W <= 8 * vec)");
+        c.edgelanes = true;
+        c.G = s.group > 0 ? s.group : 1;
+        c.L = 32;
+        c.block = 256;
+        *cfg = c;
+        return UG_OK;
+    }
     c.staged = (s.flags & UG_SCHED_TMA) ? 1 : ((s.flags & UG_SCHED_ASYNC) ? 2 : 0);
     if (c.staged) {
         // shared-memory row staging (k_svg): SV aggregation only; a misaligned A is packed first
@@ -549,7 +564,8 @@ static ug_status run(const ug_graph *g, const ug_op_info *op, const ug_schedule 
         if (ev_end) cudaEventRecord(ev_end, s);
     } else if (c.strategy == UG_TV || c.strategy == UG_WV) {
         if (ev_begin) cudaEventRecord(ev_begin, s);
-        err = launch_vertex(lw.kedge, lw.gather, ga, lw.args, c, s);
+        err = c.edgelanes ? launch_vertex_el(lw.kedge, lw.gather, ga, lw.args, c, s)
+                          : launch_vertex(lw.kedge, lw.gather, ga, lw.args, c, s);
         if (ev_end) cudaEventRecord(ev_end, s);
     } else if (c.strategy == UG_BV) {
         if (ev_begin) cudaEventRecord(ev_begin, s);
@@ -676,6 +692,7 @@ extern "C" ug_status ug_schedule_parse(const char *text, ug_schedule *out) {
         case 'P': s.flags = val ? (s.flags | UG_SCHED_PACK) : (s.flags & ~UG_SCHED_PACK); break;
         case 'M': s.flags = val ? (s.flags | UG_SCHED_TMA) : (s.flags & ~UG_SCHED_TMA); break;
         case 'A': s.flags = val ? (s.flags | UG_SCHED_ASYNC) : (s.flags & ~UG_SCHED_ASYNC); break;
+        case 'E': s.flags = val ? (s.flags | UG_SCHED_EDGELANES) : (s.flags & ~UG_SCHED_EDGELANES); break;
         default: return set_error(UG_ERR_INVALID_ARG, "bad schedule token '" + tok + "'");
         }
         pos = nxt;
@@ -697,6 +714,7 @@ extern "C" ug_status ug_schedule_format(const ug_schedule *s, char *buf, size_t 
         if (s->flags & UG_SCHED_PACK) r += "_P1";
         if (s->flags & UG_SCHED_TMA) r += "_M1";
         if (s->flags & UG_SCHED_ASYNC) r += "_A1";
+        if (s->flags & UG_SCHED_EDGELANES) r += "_E1";
     }
     std::snprintf(buf, len, "%s", r.c_str());
     return UG_OK;

@@ -52,6 +52,8 @@ def candidates(cls, F, E, quick=False):
     if cls in ("agg", "agg_bin", "agg_ext", "dot_agg"):
         c += [f"TV_G{g}_T{t}" for g in (1, 4) for t in Ts]
         c += [f"WV_G{g}_T1" for g in (1, 2, 8)]
+        if cls != "dot_agg" and F <= 32:
+            c += [f"WV_G{g}_T1_E1" for g in (1, 4)]       # lanes over in-edges (narrow F)
         c += [f"TE_G{g}_T{t}" for g in (1, 8, 32) for t in Ts if t >= 4]
         c += [f"WE_G{g}_T1" for g in (4, 32, 128)]
         vec = 4 if F % 4 == 0 else (2 if F % 2 == 0 else 1)
