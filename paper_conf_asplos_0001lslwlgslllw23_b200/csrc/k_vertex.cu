@@ -125,18 +125,25 @@ __global__ void __launch_bounds__(256) k_vertex_el(GraphArgs g, OpArgs op, int G
         for (int j = 0; j < NC; ++j)
 #pragma unroll
             for (int i = 0; i < VEC; ++i) acc[j][i] = g_init<GOP>();
-        for (int64_t k = k0 + lane; k < k1; k += 32) {
-            const int64_t src = g.col[k];
-            const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
-            const int64_t ra = op_row(op.A.type, src, v, e);
-            const int64_t rb = op_row(op.B.type, src, v, e);
+        // two in-edges per lane per step (k and k + 32: independent gathers in flight)
+        for (int64_t k = k0 + lane; k < k1; k += 64) {
+            const bool two = k + 32 < k1;
+            const int64_t kb = two ? k + 32 : k;
+            const int64_t src0 = g.col[k], src1 = g.col[kb];
+            const int64_t e0 = g.eid ? (int64_t)g.eid[k] : k, e1 = g.eid ? (int64_t)g.eid[kb] : kb;
+            const int64_t ra0 = op_row(op.A.type, src0, v, e0), rb0 = op_row(op.B.type, src0, v, e0);
+            const int64_t ra1 = op_row(op.A.type, src1, v, e1), rb1 = op_row(op.B.type, src1, v, e1);
 #pragma unroll
             for (int j = 0; j < NC; ++j) {
                 if (j * VEC < op.W) {
-                    float m[VEC];
-                    message<KE, VEC>(op, ra, ca[j], rb, cb[j], m);
+                    float m0[VEC], m1[VEC];
+                    message<KE, VEC>(op, ra0, ca[j], rb0, cb[j], m0);
+                    message<KE, VEC>(op, ra1, ca[j], rb1, cb[j], m1);
 #pragma unroll
-                    for (int i = 0; i < VEC; ++i) acc[j][i] = g_combine<GOP>(acc[j][i], m[i]);
+                    for (int i = 0; i < VEC; ++i) {
+                        acc[j][i] = g_combine<GOP>(acc[j][i], m0[i]);
+                        if (two) acc[j][i] = g_combine<GOP>(acc[j][i], m1[i]);
+                    }
                 }
             }
         }
