@@ -97,9 +97,14 @@ __device__ __forceinline__ void st_vec(float *p, const float (&r)[VEC]) {
 // ---------------------------------------------------------------- L2 cache-policy loads
 // createpolicy + ld.global.nc.L2::cache_hint: keep the gathered feature slab resident
 // (evict_last) while streaming index arrays through L2 (evict_first).
+#ifndef UG_KEEP_FRACTION
+#define UG_KEEP_FRACTION 1.0
+#endif
+#define UG_STR2(x) #x
+#define UG_STR(x) UG_STR2(x)
 __device__ __forceinline__ uint64_t l2_policy_evict_last() {
     uint64_t p;
-    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, " UG_STR(UG_KEEP_FRACTION) ";" : "=l"(p));
     return p;
 }
 __device__ __forceinline__ uint64_t l2_policy_evict_first() {

@@ -57,6 +57,8 @@ def main():
                     extra = STAGED
                 if eo == "dot" and a == "u" and b == "v":
                     extra = DOTT
+                if eo != "dot" and c == "v" and F != 18:
+                    extra = extra + ["WV_G1_T1_E1", "WV_G3_T1_E1"]      # edge-lanes (narrow F)
                 for s in SCHEDS + extra:
                     gg = gs if s in STAGED else g
                     ug.op_run(gg, eo, go, A=X, a_type=a, B=Bt, b_type=b, C=C, c_type=c, F=F, H=H, schedule=s)
