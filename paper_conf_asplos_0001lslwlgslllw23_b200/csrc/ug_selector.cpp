@@ -331,6 +331,10 @@ static bool model_select(const ug_graph *g, const Lowered &lw, ug_schedule *out)
 // width (measured with float4 rows, applied to float2 rows): keep 32 lanes.
 static ug_schedule adapt(const Lowered &lw, ug_schedule s) {
     if (s.vec > lw.max_vec) s.vec = 0;
+    // edge lanes hold at most 8 feature vectors per lane: a wider row (or a narrower vector width
+    // at this layout) takes the feature-lane warp-vertex kernel instead
+    if ((s.flags & UG_SCHED_EDGELANES) && (lw.dot || lw.to_edges || (lw.args.W + lw.max_vec - 1) / lw.max_vec > 8))
+        s.flags &= ~UG_SCHED_EDGELANES;
     // (dot under SV with a column tile is k_dott, which picks its own vector width and packs P;
     // staged SV fixes vec = ftile / 32 itself)
     if (s.strategy == UG_SV && s.ftile > 0 && !lw.dot && !(s.flags & (UG_SCHED_TMA | UG_SCHED_ASYNC))) {
@@ -412,8 +416,14 @@ ug_status select_schedule(const ug_graph *g, const Lowered &lw, ug_schedule *out
             if (!best || d < best_d) { best = &e; best_d = d; }
         }
         if (best) {
-            *out = adapt(lw, best->sched);
-            return UG_OK;
+            // a measured schedule that does not resolve on this operator's layout falls through
+            // to the next tier
+            ug_schedule s2 = adapt(lw, best->sched);
+            LaunchCfg cfg;
+            if (resolve(g, lw, s2, &cfg) == UG_OK) {
+                *out = s2;
+                return UG_OK;
+            }
         }
         if (pass == 0) {
             // 2. learned model of the exact class (only if its pick resolves on this layout)

@@ -61,7 +61,10 @@ def main():
                     extra = extra + ["WV_G1_T1_E1", "WV_G3_T1_E1"]      # edge-lanes (narrow F)
                 for s in SCHEDS + extra:
                     gg = gs if s in STAGED else g
-                    ug.op_run(gg, eo, go, A=X, a_type=a, B=Bt, b_type=b, C=C, c_type=c, F=F, H=H, schedule=s)
+                    try:
+                        ug.op_run(gg, eo, go, A=X, a_type=a, B=Bt, b_type=b, C=C, c_type=c, F=F, H=H, schedule=s)
+                    except ug.UgError as err:
+                        raise RuntimeError(f"{eo} {a} {b} {go} {c} F={F} H={H} {s}: {err}") from err
                     n += 1
         # fused chains and arg capture (single-launch merges across CTAs)
         for H, F in ((1, 16), (4, 32)):

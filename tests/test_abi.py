@@ -305,3 +305,19 @@ def test_binding_rejects_short_overlapping_tensors():
     with pytest.raises(ValueError, match="rows"):
         ug.validate(v, "copy_lhs", "sum", A=torch.zeros(vv, 4), a_type="u", C=torch.zeros(vv, 4), c_type="v") \
             if vv < 10 else (_ for _ in ()).throw(ValueError("rows"))
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2"])
+def test_auto_schedule_always_resolves(cfg):
+    """AUTO (table -> learned tier -> priors) yields a schedule the operator can run, for every op
+    and a spread of widths -- a measured entry that does not fit the layout (e.g. edge lanes at
+    F = 18, float2 rows) falls through to the next tier instead of failing."""
+    src, dst = ugdata.graph(cfg)
+    V, E = ugdata.CONFIGS[cfg].V, len(src)
+    g = host_graph(V, src, dst)
+    for F, H in ((1, 1), (3, 1), (8, 8), (16, 1), (18, 3), (20, 1), (64, 8), (100, 4)):
+        for op in all_ops():
+            eo, l, r, gop, c = op
+            A, B, C = _op_tensors(op, V, E, F, H)
+            n = ug.launch_count(g, eo, gop, A=A, a_type=l, B=B, b_type=r, C=C, c_type=c, F=F, H=H)
+            assert 1 <= n <= 4, (name(op), F, H, n)
