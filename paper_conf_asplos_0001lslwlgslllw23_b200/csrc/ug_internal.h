@@ -75,6 +75,7 @@ struct SplitPlan {
 // Kernel launchers (kernels/*.cu).  All return cudaGetLastError().
 cudaError_t launch_vertex(int kedge, int gather, const GraphArgs &g, const OpArgs &op,
                           const LaunchCfg &c, cudaStream_t s);
+cudaError_t launch_msg_el(int kedge, const GraphArgs &g, const OpArgs &op, const SplitPlan &plan, cudaStream_t s);
 cudaError_t launch_vertex_el(int kedge, int gather, const GraphArgs &g, const OpArgs &op, const LaunchCfg &c,
                              cudaStream_t s);
 cudaError_t launch_edge(int kedge, int gather, const GraphArgs &g, const OpArgs &op,

@@ -153,10 +153,22 @@ ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, La
     // SV stores through any C alignment (st_out), so its vector width is bounded by the operands
     // only; with UG_SCHED_PACK the staged copy of A is 16-byte aligned (a_vec = 4).
     c.pack = c.strategy == UG_SV && (s.flags & UG_SCHED_PACK) && lw.pack_ok;
+    if ((s.flags & UG_SCHED_EDGELANES) && c.strategy == UG_SV) {
+        // message creation with lanes over edges (k_msg_el): SV chunks, narrow messages
+        if (!lw.to_edges || lw.dot || lw.args.W > 8)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "SV _E1: message creation of an elementwise message, W <= 8");
+        c.edgelanes = true;
+        c.vec = 1;
+        c.G = s.group > 0 ? s.group : 1024;
+        c.L = 32;
+        c.block = 256;
+        *cfg = c;
+        return UG_OK;
+    }
     if (s.flags & UG_SCHED_EDGELANES) {
         // lanes over a row's in-edges (k_vertex_el): WV aggregation of an elementwise message, narrow W
         if (c.strategy != UG_WV || lw.dot || lw.to_edges)
-            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "_E1: WV aggregation of an elementwise message only");
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "_E1: WV aggregation (or SV message creation) of an elementwise message only");
         c.vec = s.vec ? s.vec : lw.max_vec;
         if (c.vec > lw.max_vec) return set_error(UG_ERR_ALIGNMENT, "forced vec wider than the operand layout allows");
         if ((lw.args.W + c.vec - 1) / c.vec > 8)
@@ -570,6 +582,12 @@ static ug_status run(const ug_graph *g, const ug_op_info *op, const ug_schedule 
     } else if (c.strategy == UG_BV) {
         if (ev_begin) cudaEventRecord(ev_begin, s);
         err = launch_block_vertex(lw.kedge, lw.gather, ga, lw.args, c, s);
+        if (ev_end) cudaEventRecord(ev_end, s);
+    } else if (c.edgelanes) {          // UG_SV message creation, lanes over edges
+        const SplitPlan *plan = nullptr;
+        if ((st = get_plan(g, c.G, &plan)) != UG_OK) return st;
+        if (ev_begin) cudaEventRecord(ev_begin, s);
+        err = launch_msg_el(lw.kedge, ga, lw.args, *plan, s);
         if (ev_end) cudaEventRecord(ev_end, s);
     } else {  // UG_SV
         const SplitPlan *plan = nullptr;

@@ -333,7 +333,8 @@ static ug_schedule adapt(const Lowered &lw, ug_schedule s) {
     if (s.vec > lw.max_vec) s.vec = 0;
     // edge lanes hold at most 8 feature vectors per lane: a wider row (or a narrower vector width
     // at this layout) takes the feature-lane warp-vertex kernel instead
-    if ((s.flags & UG_SCHED_EDGELANES) && (lw.dot || lw.to_edges || (lw.args.W + lw.max_vec - 1) / lw.max_vec > 8))
+    if ((s.flags & UG_SCHED_EDGELANES) &&
+        (lw.dot || (lw.to_edges ? lw.args.W > 8 : (lw.args.W + lw.max_vec - 1) / lw.max_vec > 8)))
         s.flags &= ~UG_SCHED_EDGELANES;
     // (dot under SV with a column tile is k_dott, which picks its own vector width and packs P;
     // staged SV fixes vec = ftile / 32 itself)

@@ -79,6 +79,8 @@ def candidates(cls, F, E, quick=False):
             c += [f"SV_G{g}_F{f}" for g in (64, 256, 512) for f in (64, 128)]     # k_dott (column tiles)
         else:   # message creation under SV: row chunks x column tiles, Dst_V operand hoisted
             c += [f"SV_G{g}_F{f}" for g in (16, 32, 64) for f in (16, 32, 64) if f <= max(16, F)]
+            if F <= 8:
+                c += [f"SV_G{g}_E1" for g in (64, 1024)]          # lanes over edges (narrow messages)
     if E > 50_000_000:   # C5: drop the schedules that take seconds (atomic per-element TE at F=602)
         c = [s for s in c if not (s.startswith("TE") and cls.startswith("agg") and "_F" not in s) and not s.startswith("TV")
              and not s.startswith("WV")]

@@ -51,3 +51,17 @@ def test_edgelanes_rejects(graph):
         ug.op_run(g, "copy_lhs", "sum", A=X[:, :8], a_type="u", C=Y[:, :8], c_type="v", F=8,
                   schedule="TV_G1_T1_E1")
     assert ug.format_schedule(ug.parse_schedule("WV_G4_T1_E1")) == "WV_G4_T1_E1"
+
+
+@pytest.mark.parametrize("mode", ["float", "int"])
+@pytest.mark.parametrize("op", [o for o in all_ops() if o[3] == "assign" and o[0] != "dot"], ids=name)
+def test_edgelanes_message_creation(graph, op, mode):
+    """SV message creation with lanes over edges ("SV_G.._E1", k_msg_el): bit-exact messages for
+    W = 1, 3 (per-head operands of width 1) and 8, on the unsorted graph (stores through eid)."""
+    V, E, src, dst, g = graph
+    for (F, H, ew) in ((1, 1, 1), (3, 3, 1), (8, 2, 8)):
+        A, B = operand_arrays(op, V, E, F, H, seed=F + 7, mode=mode, edge_width=ew)
+        ref, bound = run_oracle(op, V, src, dst, A, B, F, H)
+        for sch in ("SV_G7_E1", "SV_G1024_E1"):
+            got = run_gpu(ug, g, op, A, B, V, E, F, H, schedule=sch)
+            assert_parity(op, got, ref, bound, mode == "int", what=f"{name(op)} {sch} F={F} H={H}")
