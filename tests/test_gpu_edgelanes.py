@@ -53,12 +53,21 @@ def test_edgelanes_rejects(graph):
     assert ug.format_schedule(ug.parse_schedule("WV_G4_T1_E1")) == "WV_G4_T1_E1"
 
 
+@pytest.fixture(scope="module")
+def sorted_graph(graph):
+    V, E, src, dst, _ = graph
+    order = np.argsort(dst, kind="stable")
+    return V, E, src[order], dst[order], ug.Graph(V, src[order], dst[order])
+
+
+@pytest.mark.parametrize("kind", ["unsorted", "sorted"])
 @pytest.mark.parametrize("mode", ["float", "int"])
 @pytest.mark.parametrize("op", [o for o in all_ops() if o[3] == "assign" and o[0] != "dot"], ids=name)
-def test_edgelanes_message_creation(graph, op, mode):
+def test_edgelanes_message_creation(graph, sorted_graph, op, mode, kind):
     """SV message creation with lanes over edges ("SV_G.._E1", k_msg_el): bit-exact messages for
-    W = 1, 3 (per-head operands of width 1) and 8, on the unsorted graph (stores through eid)."""
-    V, E, src, dst, g = graph
+    W = 1, 3 (per-head operands of width 1) and 8 -- on the unsorted graph (generic form, stores
+    through eid) and the dst-sorted one (the fast form for Src_V A with none / Dst_V / Edge B)."""
+    V, E, src, dst, g = graph if kind == "unsorted" else sorted_graph
     for (F, H, ew) in ((1, 1, 1), (3, 3, 1), (8, 2, 8)):
         A, B = operand_arrays(op, V, E, F, H, seed=F + 7, mode=mode, edge_width=ew)
         ref, bound = run_oracle(op, V, src, dst, A, B, F, H)
