@@ -55,8 +55,12 @@ __device__ __forceinline__ float da_sum8(float (&v)[8], int lane) {
 
 
 
+#ifndef UG_DAW_MINB
+#define UG_DAW_MINB (VEC == 4 && NJK + NJV > 4 ? 3 : 4)   // resident CTAs per SM (r2ae: 4 beats 3 by 9-11 %)
+#endif
+
 template <int VEC, int NJK, int NJV>
-__global__ void __launch_bounds__(256, 3) k_dotattn(GraphArgs g, DotAttnArgs a, const int4 *__restrict__ chunks,
+__global__ void __launch_bounds__(256, UG_DAW_MINB) k_dotattn(GraphArgs g, DotAttnArgs a, const int4 *__restrict__ chunks,
                                                     int n_chunks, float *__restrict__ scratch, int64_t sld) {
     const int lane = threadIdx.x & 31;
     const int u = (int)(blockIdx.x * 8 + (threadIdx.x >> 5));
@@ -173,23 +177,31 @@ __global__ void __launch_bounds__(256, 3) k_dotattn(GraphArgs g, DotAttnArgs a, 
     }
 }
 
-// Packed heads (Dk = Dv = D, w = D / VEC a power of two, H * w <= 32): one unit = one SV chunk
-// with ALL its heads, L = pow2(H * w) lanes, lane = h * w + i owning features h*D + i*VEC.  A
+// Packed heads (Dk = Dv = D, w = D / VEC a power of two <= 16): one unit = one SV chunk with a
+// group of 32 / w heads (all H when H * w <= 32), L = min(32, pow2(H * w)) lanes, lane = h * w + i
+// of the group owning features h*D + i*VEC; units are group-major (the groups' K / V column
+// slabs are walked one after another, as the SV column tiles).  A
 // head's score is reduced over its w lanes by a log2(w)-step xor butterfly that leaves it in all
 // of them, so every lane runs the online softmax of its own head -- no idle lanes for small
 // heads (C2: D = 8, w = 2) and no broadcast.  UE in-edges per step.
+#ifndef UG_DAH_MINB
+#define UG_DAH_MINB 4   // resident CTAs per SM the register budget is sized for
+#endif
+
 template <int VEC, int UE>
-__global__ void __launch_bounds__(256) k_dotattn_heads(GraphArgs g, DotAttnArgs a, const int4 *__restrict__ chunks,
-                                                       int n_chunks, int L_log2, int w_log2,
+__global__ void __launch_bounds__(256, UG_DAH_MINB) k_dotattn_heads(GraphArgs g, DotAttnArgs a, const int4 *__restrict__ chunks,
+                                                       int n_chunks, int n_units, int L_log2, int w_log2,
                                                        float *__restrict__ scratch, int64_t sld) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int L = 1 << L_log2, w = 1 << w_log2;
     const int lane = (int)(t & (L - 1));
-    const int64_t u = t >> L_log2;
-    if (u >= n_chunks) return;                    // whole units: a unit's lanes leave together
+    const int64_t ut = t >> L_log2;
+    if (ut >= n_units) return;                    // whole units: a unit's lanes leave together
+    const int grp = n_units == n_chunks ? 0 : (int)ut / n_chunks;   // head group (0: all heads fit one unit)
+    const int u = (int)ut - grp * n_chunks;
     const int wl = threadIdx.x & 31;
     const unsigned umask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << (wl & ~(L - 1)));
-    const int h = lane >> w_log2, i = lane & (w - 1);
+    const int h = ((grp << L_log2) + lane) >> w_log2, i = lane & (w - 1);
     const bool active = h < a.H;
     const int hh = active ? h : 0;
     const int f = hh * a.Dk + i * VEC;            // Dk == Dv
@@ -321,27 +333,34 @@ cudaError_t launch_dotattn_tail(const GraphArgs &g, const DotAttnArgs &a, const 
 
 cudaError_t launch_dotattn(const GraphArgs &g, const DotAttnArgs &a, int vec, const SplitPlan &plan,
                            float *scratch, int64_t sld, cudaStream_t s) {
-    const int njk = (int)cdiv(a.Dk, 32 * vec), njv = (int)cdiv(a.Dv, 32 * vec);
     const int64_t units = plan.n_chunks * (int64_t)a.H;
     if (units == 0) return cudaSuccess;
     cudaError_t err = cudaSuccess;
     const int wl = a.Dk / vec;
-    static const bool force_wide = std::getenv("UG_DOTATTN_WIDE") != nullptr;   // A/B switch
-    // packed heads when a head spans <= 8 lanes (<= 3 butterfly steps per edge); wider heads reduce
-    // 8 edges at once by the transposed butterfly (C4 H = 1, D = 128: 303 -> 226 us; H = 8: packed
-    // 236 us vs 1,288 us; profiles/r2/ab_r2t.log)
-    if (!force_wide && a.Dk == a.Dv && a.Dk % vec == 0 && (wl & (wl - 1)) == 0 && wl <= 8 &&
-        (int64_t)a.H * wl <= 32) {
-        // packed heads: one unit per chunk with all H heads (k_dotattn_heads)
+    static const bool force_wide = std::getenv("UG_DOTATTN_WIDE") != nullptr;   // A/B switches
+    static const int pack_wl = std::getenv("UG_DOTATTN_PACK_WL") ? std::atoi(std::getenv("UG_DOTATTN_PACK_WL")) : 16;
+    // packed heads when a head spans <= 16 lanes (<= 4 butterfly steps per edge; r2ag: C4 H = 1,
+    // D = 64 152 -> 133 us, H = 2 D = 64 281 -> 234 us at 16 vs 8); wider heads reduce 8 edges at
+    // once by the transposed butterfly (C4 H = 1, D = 128: 303 -> 226 us; H = 8: packed 236 us vs
+    // 1,288 us; profiles/r2/ab_r2t.log)
+    if (!force_wide && a.Dk == a.Dv && a.Dk % vec == 0 && (wl & (wl - 1)) == 0 && wl <= pack_wl) {
+        // packed heads: one unit per (head group, chunk) (k_dotattn_heads)
         int L = 1;
-        while (L < a.H * wl) L <<= 1;
-        const int64_t grid = cdiv(plan.n_chunks * (int64_t)L, 256);
+        while (L < a.H * wl && L < 32) L <<= 1;
+        const int64_t n_units = plan.n_chunks * cdiv((int64_t)a.H * wl, L);
+        if (n_units * L >= (1ll << 31)) return cudaErrorInvalidValue;
+        const int64_t grid = cdiv(n_units * L, 256);
         const int4 *ch = reinterpret_cast<const int4 *>(plan.d_chunk);
         UG_DISPATCH_VEC(vec, VEC,
-            k_dotattn_heads<VEC, 4><<<(unsigned)grid, 256, 0, s>>>(g, a, ch, (int)plan.n_chunks, ilog2(L),
-                                                                   ilog2(wl), scratch, sld));
+            k_dotattn_heads<VEC, 4><<<(unsigned)grid, 256, 0, s>>>(g, a, ch, (int)plan.n_chunks, (int)n_units,
+                                                                   ilog2(L), ilog2(wl), scratch, sld));
     } else {
-        err = launch_dotattn_wide(g, a, vec, njk, njv, plan, scratch, sld, s);
+        // one warp per head: the narrowest vector that still gives every lane a chunk (D = 64:
+        // float2 x 32 lanes rather than float4 x 16 lanes with half the warp idle)
+        int vw = vec;
+        while (vw > 1 && (a.Dk < 32 * vw || a.Dv < 32 * vw) && cdiv(a.Dk, 16 * vw) <= 4 && cdiv(a.Dv, 16 * vw) <= 4)
+            vw >>= 1;
+        err = launch_dotattn_wide(g, a, vw, (int)cdiv(a.Dk, 32 * vw), (int)cdiv(a.Dv, 32 * vw), plan, scratch, sld, s);
     }
     if (err == cudaSuccess) err = cudaGetLastError();
     if (err != cudaSuccess) return err;

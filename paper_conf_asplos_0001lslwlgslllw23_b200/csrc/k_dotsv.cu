@@ -17,8 +17,12 @@
 
 namespace ug {
 
+#ifndef UG_DOTSV_MINB
+#define UG_DOTSV_MINB 4   // resident CTAs per SM the register budget is sized for
+#endif
+
 template <int GOP, int VEC, int NJ>
-__global__ void __launch_bounds__(256, 4) k_dotsv(GraphArgs g, OpArgs op, bool a_is_src, const int4 *__restrict__ chunks,
+__global__ void __launch_bounds__(256, UG_DOTSV_MINB) k_dotsv(GraphArgs g, OpArgs op, bool a_is_src, const int4 *__restrict__ chunks,
                                                   int64_t n_chunks, int L_log2, int w_log2,
                                                   float *__restrict__ scratch, int64_t sld) {
     constexpr int UE = NJ * VEC >= 16 ? 1 : 16 / (NJ * VEC);   // in-edges per step

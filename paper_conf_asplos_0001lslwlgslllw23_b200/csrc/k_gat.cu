@@ -145,8 +145,12 @@ __device__ __forceinline__ void gat_store(const GatArgs &a, int64_t v, int f, co
 // unit order.  Chunks of rows longer than the chunk size write their (max, den, acc) state to
 // scratch; the slice that completes a row's last chunk (per-row arrival counter) merges the
 // states in chunk order -- deterministic, one launch, no atomics on the data.
+#ifndef UG_GAT_MINB
+#define UG_GAT_MINB 1   // resident CTAs per SM the register budget is sized for
+#endif
+
 template <int VEC, int U, bool ATTN>
-__global__ void __launch_bounds__(256) k_gat(GraphArgs g, GatArgs a, int L_log2, int n_tiles,
+__global__ void __launch_bounds__(256, UG_GAT_MINB) k_gat(GraphArgs g, GatArgs a, int L_log2, int n_tiles,
                                              const int4 *__restrict__ chunks, int64_t n_chunks,
                                              const int4 *__restrict__ split, const int32_t *__restrict__ slot_row,
                                              float *sacc, float *sst, int64_t sld, int64_t nfc,

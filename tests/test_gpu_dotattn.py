@@ -39,7 +39,8 @@ def _check(V, src, dst, H, Dk, Dv, seed, g=None, attn=True, scale=None):
 
 
 @pytest.mark.parametrize("H,Dk,Dv", [(1, 16, 16), (8, 8, 8), (2, 64, 32), (4, 3, 5), (1, 128, 128), (1, 256, 64),
-                                     (3, 30, 50), (1, 512, 512)])
+                                     (3, 30, 50), (1, 512, 512),
+                                     (4, 64, 64), (1, 96, 96), (1, 64, 128), (5, 32, 32), (3, 64, 64)])
 def test_dotattn_random_multigraphs(H, Dk, Dv):
     for seed in range(3):
         V = 60 + 50 * seed
@@ -47,7 +48,7 @@ def test_dotattn_random_multigraphs(H, Dk, Dv):
         _check(V, src, dst, H, Dk, Dv, 50 + seed)
 
 
-@pytest.mark.parametrize("H,Dk,Dv", [(1, 16, 16), (8, 8, 8), (2, 128, 64)])
+@pytest.mark.parametrize("H,Dk,Dv", [(1, 16, 16), (8, 8, 8), (2, 128, 64), (4, 64, 64), (5, 32, 32)])
 def test_dotattn_hub_split_rows(H, Dk, Dv):
     V = 3001
     s = np.concatenate([np.arange(1, V), np.arange(V)]).astype(np.int32)
@@ -55,7 +56,8 @@ def test_dotattn_hub_split_rows(H, Dk, Dv):
     _check(V, s, d, H, Dk, Dv, 7)
 
 
-@pytest.mark.parametrize("cfg,H,F", [("C2", 8, 64), ("C2", 1, 16), ("C4", 8, 128), ("C4", 1, 128)])
+@pytest.mark.parametrize("cfg,H,F", [("C2", 8, 64), ("C2", 1, 16), ("C4", 8, 128), ("C4", 1, 128),
+                                         ("C4", 4, 256), ("C4", 1, 64)])
 def test_dotattn_configs(cfg, H, F):
     c = ugdata.CONFIGS[cfg]
     src, dst = ugdata.graph(cfg)
