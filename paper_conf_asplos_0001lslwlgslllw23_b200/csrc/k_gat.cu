@@ -72,23 +72,40 @@ __device__ __forceinline__ void gat_walk(const GraphArgs &g, const GatArgs &a, i
     // padding slots read row 0 (cache-hot) and are masked by t = -inf: no branches
     const float *zb = a.z + (active ? f : 0);
     const float *eb = a.el + h;
+#ifndef UG_GAT_HINTS
+#define UG_GAT_HINTS 0   // L2 evict hints on the walk's loads: +24 registers, r2aj/r2ak: slower at every budget
+#endif
+#if UG_GAT_HINTS
+    const uint64_t keep = l2_policy_evict_last(), stream = l2_policy_evict_first();
+#define UG_GAT_COL(k) ldg_i32_hint(g.col + (k), stream)
+#else
+#define UG_GAT_COL(k) __ldg(g.col + (k))
+#endif
     int32_t nxt[U];
 #pragma unroll
-    for (int q = 0; q < U; ++q) nxt[q] = k0 + q < k1 ? __ldg(g.col + k0 + q) : -1;
+    for (int q = 0; q < U; ++q) nxt[q] = k0 + q < k1 ? UG_GAT_COL(k0 + q) : -1;
     for (int k = k0; k < k1; k += U) {
         int32_t cur[U];
 #pragma unroll
         for (int q = 0; q < U; ++q) {
             cur[q] = nxt[q];
-            nxt[q] = k + U + q < k1 ? __ldg(g.col + k + U + q) : -1;
+            nxt[q] = k + U + q < k1 ? UG_GAT_COL(k + U + q) : -1;
         }
         float t[U], zr[U][VEC];
 #pragma unroll
         for (int q = 0; q < U; ++q) {
-            const int64_t u = cur[q] < 0 ? 0 : cur[q];
-            t[q] = __ldg(eb + u * a.ld_el);
-            ldg_vec<VEC>(zb + u * a.ld_z, zr[q]);
+            const uint32_t u = cur[q] < 0 ? 0u : (uint32_t)cur[q];
+#if UG_GAT_HINTS
+            float tt[1];
+            ldg_vec_hint<1>(eb + (int64_t)u * a.ld_el, tt, keep);
+            t[q] = tt[0];
+            ldg_vec_hint<VEC>(zb + (int64_t)u * a.ld_z, zr[q], keep);
+#else
+            t[q] = __ldg(eb + (int64_t)u * a.ld_el);
+            ldg_vec<VEC>(zb + (int64_t)u * a.ld_z, zr[q]);
+#endif
         }
+#undef UG_GAT_COL
         float mn = st.m;
 #pragma unroll
         for (int q = 0; q < U; ++q) {
@@ -145,12 +162,11 @@ __device__ __forceinline__ void gat_store(const GatArgs &a, int64_t v, int f, co
 // unit order.  Chunks of rows longer than the chunk size write their (max, den, acc) state to
 // scratch; the slice that completes a row's last chunk (per-row arrival counter) merges the
 // states in chunk order -- deterministic, one launch, no atomics on the data.
-#ifndef UG_GAT_MINB
-#define UG_GAT_MINB 1   // resident CTAs per SM the register budget is sized for
-#endif
-
-template <int VEC, int U, bool ATTN>
-__global__ void __launch_bounds__(256, UG_GAT_MINB) k_gat(GraphArgs g, GatArgs a, int L_log2, int n_tiles,
+// MB = resident CTAs per SM the register budget is sized for: 6 (40 registers) for float4 slices of
+// large graphs, 1 (no cap, 48) otherwise -- r2al: C4 H = 8 F = 128 148.8 -> 128.3 us, C3 H = 4
+// F = 64 224 -> 190 us, but C2 14.7 -> 15.7 us, hence by grid size
+template <int VEC, int U, bool ATTN, int MB>
+__global__ void __launch_bounds__(256, MB) k_gat(GraphArgs g, GatArgs a, int L_log2, int n_tiles,
                                              const int4 *__restrict__ chunks, int64_t n_chunks,
                                              const int4 *__restrict__ split, const int32_t *__restrict__ slot_row,
                                              float *sacc, float *sst, int64_t sld, int64_t nfc,
@@ -229,15 +245,20 @@ cudaError_t launch_gat(const GraphArgs &g, const GatArgs &a, int vec, int L, con
     const int L_log2 = ilog2(L);
     const int4 *chunks = reinterpret_cast<const int4 *>(plan.d_chunk);
     const int4 *split = reinterpret_cast<const int4 *>(plan.d_split);
+    const bool big = grid >= 4096;
+#define UG_GAT_LAUNCH(ATTN_, MB_)                                                                               \
+    k_gat<VEC, (VEC == 4 ? 4 : 8), ATTN_, MB_><<<(unsigned)grid, block, 0, s>>>(                               \
+        g, a, L_log2, n_tiles, chunks, plan.n_chunks, split, slot_row, sacc, sst, sld, nfc, counters)
     UG_DISPATCH_VEC(vec, VEC, {
-        constexpr int U = VEC == 4 ? 4 : 8;
-        if (a.attn)
-            k_gat<VEC, U, true><<<(unsigned)grid, block, 0, s>>>(g, a, L_log2, n_tiles, chunks, plan.n_chunks, split,
-                                                                 slot_row, sacc, sst, sld, nfc, counters);
-        else
-            k_gat<VEC, U, false><<<(unsigned)grid, block, 0, s>>>(g, a, L_log2, n_tiles, chunks, plan.n_chunks, split,
-                                                                  slot_row, sacc, sst, sld, nfc, counters);
+        if constexpr (VEC == 4) {
+            if (a.attn) { if (big) UG_GAT_LAUNCH(true, 6); else UG_GAT_LAUNCH(true, 1); }
+            else { if (big) UG_GAT_LAUNCH(false, 6); else UG_GAT_LAUNCH(false, 1); }
+        } else {
+            if (a.attn) UG_GAT_LAUNCH(true, 1);
+            else UG_GAT_LAUNCH(false, 1);
+        }
     });
+#undef UG_GAT_LAUNCH
     return cudaGetLastError();
 }
 
