@@ -55,6 +55,16 @@ __device__ __forceinline__ float da_sum8(float (&v)[8], int lane) {
 
 
 
+// column-index prefetch (the next batch's col_idx loads overlap this batch's row gathers), per
+// kernel form -- r2an: packed heads C3 H = 4 D = 16 289 -> 269 us, C4 H = 8 199 -> 190 us; one warp
+// per head C4 H = 1 D = 128 203 -> 209 us, so off there
+#ifndef UG_DAH_PF
+#define UG_DAH_PF 1
+#endif
+#ifndef UG_DAW_PF
+#define UG_DAW_PF 0
+#endif
+
 #ifndef UG_DAW_MINB
 #define UG_DAW_MINB (VEC == 4 && NJK + NJV > 4 ? 3 : 4)   // resident CTAs per SM (r2ae: 4 beats 3 by 9-11 %)
 #endif
@@ -93,11 +103,24 @@ __global__ void __launch_bounds__(256, UG_DAW_MINB) k_dotattn(GraphArgs g, DotAt
 #pragma unroll
         for (int i = 0; i < VEC; ++i) acc[j][i] = 0.0f;
     const int k1 = ch.z;
+    const int last = k1 - 1;
+    // the next batch's column indices are loaded while this batch is gathered (UG_DAW_PF)
+    uint32_t s_pf[8];
+    if (UG_DAW_PF && ch.y < k1) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) s_pf[i] = (uint32_t)ldg_i32_hint(g.col + min(ch.y + i, last), stream);
+    }
     for (int k0 = ch.y; k0 < k1; k0 += 8) {
-        const int last = k1 - 1;
         uint32_t s[8];
 #pragma unroll
-        for (int i = 0; i < 8; ++i) s[i] = (uint32_t)ldg_i32_hint(g.col + min(k0 + i, last), stream);
+        for (int i = 0; i < 8; ++i) {
+            if (UG_DAW_PF) {
+                s[i] = s_pf[i];
+                s_pf[i] = (uint32_t)ldg_i32_hint(g.col + min(k0 + 8 + i, last), stream);
+            } else {
+                s[i] = (uint32_t)ldg_i32_hint(g.col + min(k0 + i, last), stream);
+            }
+        }
         float p[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
@@ -218,11 +241,23 @@ __global__ void __launch_bounds__(256, UG_DAH_MINB) k_dotattn_heads(GraphArgs g,
 #pragma unroll
     for (int c = 0; c < VEC; ++c) acc[c] = 0.0f;
     const int k1 = ch.z;
+    const int last = k1 - 1;
+    uint32_t s_pf[UE];
+    if (UG_DAH_PF && ch.y < k1) {
+#pragma unroll
+        for (int e = 0; e < UE; ++e) s_pf[e] = (uint32_t)ldg_i32_hint(g.col + min(ch.y + e, last), stream);
+    }
     for (int k0 = ch.y; k0 < k1; k0 += UE) {
-        const int last = k1 - 1;
         uint32_t sidx[UE];
 #pragma unroll
-        for (int e = 0; e < UE; ++e) sidx[e] = (uint32_t)ldg_i32_hint(g.col + min(k0 + e, last), stream);
+        for (int e = 0; e < UE; ++e) {
+            if (UG_DAH_PF) {
+                sidx[e] = s_pf[e];
+                s_pf[e] = (uint32_t)ldg_i32_hint(g.col + min(k0 + UE + e, last), stream);
+            } else {
+                sidx[e] = (uint32_t)ldg_i32_hint(g.col + min(k0 + e, last), stream);
+            }
+        }
         float kx[UE][VEC], vx[UE][VEC];
 #pragma unroll
         for (int e = 0; e < UE; ++e) {

@@ -76,11 +76,29 @@ __global__ void __launch_bounds__(256, UG_DOTSV_MINB) k_dotsv(GraphArgs g, OpArg
     };
     int k = ch.y;                               // CSR positions are int32
     const int k1 = ch.z;
+    // the next step's column indices are loaded while this step's rows are gathered (UG_DOTSV_PF;
+    // r2an: C4 u_dot_v F = 128 79.8 -> 69.6 us, C3 276 -> 244 us, C4 u_dot_v_sum 82 -> 74 us)
+#ifndef UG_DOTSV_PF
+#define UG_DOTSV_PF 1
+#endif
+    constexpr bool PF = UG_DOTSV_PF && UE <= 4;
+    int32_t s_pf[UE];
+    if (PF && k + UE <= k1) {
+#pragma unroll
+        for (int e = 0; e < UE; ++e) s_pf[e] = ldg_i32_hint(g.col + k + e, stream);
+    }
     for (; k + UE <= k1; k += UE) {
         float p[UE][NJ][VEC];
         int64_t s[UE];
 #pragma unroll
-        for (int e = 0; e < UE; ++e) s[e] = ldg_i32_hint(g.col + k + e, stream);
+        for (int e = 0; e < UE; ++e) {
+            if (PF) {
+                s[e] = s_pf[e];
+                s_pf[e] = ldg_i32_hint(g.col + min(k + UE + e, k1 - 1), stream);
+            } else {
+                s[e] = ldg_i32_hint(g.col + k + e, stream);
+            }
+        }
 #pragma unroll
         for (int e = 0; e < UE; ++e) {
 #pragma unroll

@@ -45,12 +45,38 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
     float bconst[VEC];
     if constexpr (BM == 1) fetch<VEC>(op.B, v, cb, bconst);
     const int64_t kl = k1 - 1;
+    // PF: the next group's column indices are loaded while this group's rows are gathered, so a
+    // group costs one dependent L2 round trip (row) instead of two (col_idx, then row).  Off: it
+    // measured slower here (r2an: C3 u_mul_e_sum 285 -> 293 us, C5 21.0 -> 24.3 ms; copy with
+    // 6-7 CTAs / SM to make room 215 -> 244 us) -- unlike k_dotsv / k_dotattn_heads, where it wins
+#ifndef UG_PF_BM2
+#define UG_PF_BM2 0
+#endif
+#ifndef UG_PF_BM0
+#define UG_PF_BM0 0
+#endif
+    constexpr bool PF = VEC == 4 && ((BM == 2 && UG_PF_BM2) || ((BM == 0 || BM == 1) && UG_PF_BM0));
+    uint32_t s_pf[UF];
+    if constexpr (PF) {
+        if (k + UF <= k1) {                          // (empty rows: col[k1 - 1] may not exist)
+#pragma unroll
+            for (int q = 0; q < UF; ++q) s_pf[q] = (uint32_t)ldg_i32_hint(g.col + k + q, stream);
+        }
+    }
     auto group = [&](auto pred_tag, auto n_tag) {
         constexpr bool PRED = decltype(pred_tag)::value;
         constexpr int UF = decltype(n_tag)::value;
         uint32_t s[UF];
+        if constexpr (PF && !PRED) {
 #pragma unroll
-        for (int q = 0; q < UF; ++q) s[q] = (uint32_t)ldg_i32_hint(g.col + (PRED ? min(k + q, kl) : k + q), stream);
+            for (int q = 0; q < UF; ++q) {
+                s[q] = s_pf[q];
+                s_pf[q] = (uint32_t)ldg_i32_hint(g.col + min(k + UF + q, kl), stream);
+            }
+        } else {
+#pragma unroll
+            for (int q = 0; q < UF; ++q) s[q] = (uint32_t)ldg_i32_hint(g.col + (PRED ? min(k + q, kl) : k + q), stream);
+        }
         float m[UF][VEC];
 #pragma unroll
         for (int q = 0; q < UF; ++q) ldg_vec_hint<VEC>(Ab + (s[q] * lda + fo), m[q], keep);
