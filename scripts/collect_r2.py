@@ -1,5 +1,5 @@
 #!/usr/bin/env python
-"""Copy one evidence run of scripts/gpu_r2_final.sh (gpurun_out/*_<tag>*) into profiles/ and
+"""Copy one evidence run of scripts/gpu_evidence.sh (gpurun_out/*_<tag>*) into profiles/ and
 summarise it (run here, on the CPU host):
 
     python scripts/collect_r2.py r2fa
