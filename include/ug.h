@@ -126,11 +126,14 @@ typedef struct {
                              by TMA (cp.async.bulk.tensor tile::gather4, issued by one lane per
                              warp) into a per-warp ring of shared-memory stages completed on
                              mbarriers, instead of into registers                                */
-#define UG_SCHED_EDGELANES 8  /* WV aggregation with W / vec <= 8 ("_E1"): the 32 lanes of a warp take
-                                 a destination row's in-edges round-robin and reduce all its
-                                 features in registers, then combine by an xor butterfly -- one
-                                 launch, owner computes; for narrow features on small, skewed
-                                 graphs, where feature lanes leave most lanes idle             */
+#define UG_SCHED_EDGELANES 8  /* WV / TV aggregation with W / vec <= 8 ("_E1"): the lanes of a row
+                                 (WV_Gg_T1_E1: a warp; TV_Gg_Tt_E1, t in {8, 16}: t lanes, 32 / t
+                                 rows per warp) take its in-edges round-robin and reduce all its
+                                 features in registers, then combine by a transposed butterfly --
+                                 one launch, owner computes; for narrow features on small, skewed
+                                 graphs, where feature lanes leave most lanes idle.  SV message
+                                 creation ("SV_Gg_E1", W <= 8): one warp per chunk, lanes over
+                                 its consecutive in-edges                                       */
 #define UG_SCHED_ASYNC 4  /* SV aggregation only ("_A1"): the same ring filled by cp.async
                              (LDGSTS, each lane its own features of the group's four rows).
                              Both staged forms: ftile = 32 * vec columns (128 / 64 / 32), a

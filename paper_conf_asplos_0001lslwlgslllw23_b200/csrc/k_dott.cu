@@ -81,11 +81,31 @@ __global__ void __launch_bounds__(256, UG_DOTT_MINB) k_dott(GraphArgs g, OpArgs 
     const int k1 = ch.z;
     // a batch: 8 column indices, then 8 row gathers (UG_DOTT_PIPE=1 issues the next batch's before
     // reducing the current one -- measured slower, kept for A/B)
-    auto load_batch = [&](int k, float (&x)[8][VEC]) {
-        const int last = k1 - 1;
-        uint32_t s[8];
+    // UG_DOTT_PF: the next batch's 8 column indices are loaded while this batch's rows are gathered
+    // (one dependent L2 round trip per batch instead of two; it won in k_dotsv, r2an)
+#ifndef UG_DOTT_PF
+#define UG_DOTT_PF 0
+#endif
+    const int last = k1 - 1;
+    uint32_t s_pf[8];
+    if constexpr (UG_DOTT_PF) {
+        if (ch.y < k1) {                              // (an empty chunk has no col[k1 - 1])
 #pragma unroll
-        for (int i = 0; i < 8; ++i) s[i] = (uint32_t)ldg_i32_hint(g.col + min(k + i, last), stream);
+            for (int i = 0; i < 8; ++i) s_pf[i] = (uint32_t)ldg_i32_hint(g.col + min(ch.y + i, last), stream);
+        }
+    }
+    auto load_batch = [&](int k, float (&x)[8][VEC]) {
+        uint32_t s[8];
+        if constexpr (UG_DOTT_PF) {
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                s[i] = s_pf[i];
+                s_pf[i] = (uint32_t)ldg_i32_hint(g.col + min(k + 8 + i, last), stream);
+            }
+        } else {
+#pragma unroll
+            for (int i = 0; i < 8; ++i) s[i] = (uint32_t)ldg_i32_hint(g.col + min(k + i, last), stream);
+        }
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
             // branch-free: every lane loads a full vector from a valid address (an inactive lane

@@ -98,37 +98,67 @@ cudaError_t launch_vertex(int kedge, int gather, const GraphArgs &g, const OpArg
     return cudaGetLastError();
 }
 
-// Edge-lanes warp-vertex ("WV_..._E1", round 2): for narrow features (W / VEC <= 8 chunks) the
-// lanes of a warp split a destination row's IN-EDGES instead of its features -- lane l takes
-// edges k0 + l, k0 + l + 32, ... and reduces every feature of its messages in registers, then an
-// xor butterfly over the 32 lanes combines them (owner computes: one launch, no atomics, no
-// init).  A row of in-degree d costs ceil(d / 32) dependent gather steps instead of d / UF, which
-// is what bounds small, skewed graphs (C1 / C2) under the feature-lane schedules.
-template <int KE, int GOP, int VEC, int NC>
+// Reduce N values (N a power of two) over the P lanes of a lane segment (P a power of two <= 32,
+// segments aligned in the warp) with gather_op GOP, by a transposed butterfly: at offsets P/2,
+// P/4, ... each lane sends half of its remaining values and keeps the other half.  After it,
+// lane l of the segment holds in v[0 .. max(N / P, 1)) the totals of values
+// (l >> (log2 P - log2 N)) when N <= P, or l * (N / P) + i when N > P (contiguous columns).
+// N - 1 + log2 P - log2 N shuffles for N <= P, instead of N log2 P for N separate butterflies.
+// Fixed tree: deterministic.  Every lane of the warp must call it.
+template <int GOP, int N, int P>
+__device__ __forceinline__ void seg_reduce_transposed(float (&v)[N], int lane) {
+#pragma unroll
+    for (int n = N, o = P / 2; n > 1 && o > 0; n >>= 1, o >>= 1) {
+        const bool up = lane & o;
+#pragma unroll
+        for (int i = 0; i < n / 2; ++i) {
+            const float send = up ? v[i] : v[i + n / 2];
+            const float keep = up ? v[i + n / 2] : v[i];
+            v[i] = g_combine<GOP>(keep, __shfl_xor_sync(0xffffffffu, send, o));
+        }
+    }
+    if constexpr (N < P) {
+#pragma unroll
+        for (int o = P / N / 2; o > 0; o >>= 1) v[0] = g_combine<GOP>(v[0], __shfl_xor_sync(0xffffffffu, v[0], o));
+    }
+}
+
+// Edge-lanes vertex schedules ("WV_Gg_T1_E1": P = 32 lanes per row; "TV_Gg_Tp_E1": P = p lanes,
+// 32 / p rows per warp; round 2): for narrow features (W / VEC <= 8 chunks) the P lanes of a row
+// split its IN-EDGES instead of its features -- lane l takes edges k0 + l, k0 + l + P, ... and
+// reduces every feature of its messages in registers; a transposed butterfly over the P lanes
+// then combines them (owner computes: one launch, no atomics, no init).  A row of in-degree d
+// costs ceil(d / 2P) dependent gather steps instead of d / UF, which is what bounds small, skewed
+// graphs (C1 / C2) under the feature-lane schedules; P < 32 packs several light rows per warp
+// (fewer waves on graphs with more rows than resident warps, e.g. C2).
+template <int KE, int GOP, int VEC, int NC, int P>
 __global__ void __launch_bounds__(256) k_vertex_el(GraphArgs g, OpArgs op, int G) {
-    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    constexpr int N = NC * VEC;                       // values per lane (a power of two)
+    constexpr int NOUT = N > P ? N / P : 1;           // totals a lane holds after the reduction
+    const int64_t seg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / P;   // row group
     const int lane = threadIdx.x & 31;
-    const int64_t v0 = warp * G;
-    if (v0 >= g.V) return;                            // whole warps leave together
-    const int64_t v_end = min(g.V, v0 + (int64_t)G);
+    const int sl = lane & (P - 1);                    // lane within the row's segment
+    const int64_t warp0 = (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * (32 / P);
+    if (warp0 * G >= g.V) return;                     // whole warps leave together
     int64_t ca[NC], cb[NC];
 #pragma unroll
     for (int j = 0; j < NC; ++j) {
         ca[j] = op_col(op.A, min(j * VEC, op.W - 1));
         cb[j] = op_col(op.B, min(j * VEC, op.W - 1));
     }
-    for (int64_t v = v0; v < v_end; ++v) {
-        const int64_t k0 = (int64_t)g.row_ptr[v] - g.rp_base;
-        const int64_t k1 = (int64_t)g.row_ptr[v + 1] - g.rp_base;
-        float acc[NC][VEC];
+    for (int r = 0; r < G; ++r) {
+        const int64_t v = seg * G + r;
+        if ((warp0 * G + r) >= g.V) break;            // warp-uniform: the warp's first row group
+        const bool live = v < g.V;
+        const int64_t k0 = live ? (int64_t)g.row_ptr[v] - g.rp_base : 0;
+        const int64_t k1 = live ? (int64_t)g.row_ptr[v + 1] - g.rp_base : 0;
+        float acc[N];
 #pragma unroll
-        for (int j = 0; j < NC; ++j)
-#pragma unroll
-            for (int i = 0; i < VEC; ++i) acc[j][i] = g_init<GOP>();
-        // two in-edges per lane per step (k and k + 32: independent gathers in flight)
-        for (int64_t k = k0 + lane; k < k1; k += 64) {
-            const bool two = k + 32 < k1;
-            const int64_t kb = two ? k + 32 : k;
+        for (int j = 0; j < N; ++j) acc[j] = g_init<GOP>();
+        // two in-edges per lane per step (k and k + P: independent gathers in flight)
+        for (int64_t k = k0 + sl; k < k1; k += 2 * P) {
+            const bool two = k + P < k1;
+            const int64_t kb = two ? k + P : k;
             const int64_t src0 = g.col[k], src1 = g.col[kb];
             const int64_t e0 = g.eid ? (int64_t)g.eid[k] : k, e1 = g.eid ? (int64_t)g.eid[kb] : kb;
             const int64_t ra0 = op_row(op.A.type, src0, v, e0), rb0 = op_row(op.B.type, src0, v, e0);
@@ -141,27 +171,25 @@ __global__ void __launch_bounds__(256) k_vertex_el(GraphArgs g, OpArgs op, int G
                     message<KE, VEC>(op, ra1, ca[j], rb1, cb[j], m1);
 #pragma unroll
                     for (int i = 0; i < VEC; ++i) {
-                        acc[j][i] = g_combine<GOP>(acc[j][i], m0[i]);
-                        if (two) acc[j][i] = g_combine<GOP>(acc[j][i], m1[i]);
+                        acc[j * VEC + i] = g_combine<GOP>(acc[j * VEC + i], m0[i]);
+                        if (two) acc[j * VEC + i] = g_combine<GOP>(acc[j * VEC + i], m1[i]);
                     }
                 }
             }
         }
-#pragma unroll
-        for (int off = 16; off > 0; off >>= 1)
-#pragma unroll
-            for (int j = 0; j < NC; ++j)
-#pragma unroll
-                for (int i = 0; i < VEC; ++i)
-                    acc[j][i] = g_combine<GOP>(acc[j][i], __shfl_xor_sync(0xffffffffu, acc[j][i], off));
+        seg_reduce_transposed<GOP, N, P>(acc, lane);
         const int64_t deg = k1 - k0;
+        if (live) {
+            if constexpr (N <= P) {
+                constexpr int SH = (P >= 32 ? 5 : P >= 16 ? 4 : P >= 8 ? 3 : P >= 4 ? 2 : P >= 2 ? 1 : 0) -
+                                   (N >= 32 ? 5 : N >= 16 ? 4 : N >= 8 ? 3 : N >= 4 ? 2 : N >= 2 ? 1 : 0);
+                const int col = sl >> SH;
+                if ((sl & ((1 << SH) - 1)) == 0 && col < op.W) op.C[v * op.c_ld + col] = g_finalize<GOP>(acc[0], deg);
+            } else {
+                const int c0 = sl * NOUT;
 #pragma unroll
-        for (int j = 0; j < NC; ++j) {
-            if (lane == j && j * VEC < op.W) {        // lane j stores chunk j
-                float o[VEC];
-#pragma unroll
-                for (int i = 0; i < VEC; ++i) o[i] = g_finalize<GOP>(acc[j][i], deg);
-                st_out<VEC>(op.C + v * op.c_ld + j * VEC, o, op.W - j * VEC, op.c_vec);
+                for (int i = 0; i < NOUT; ++i)
+                    if (c0 + i < op.W) op.C[v * op.c_ld + c0 + i] = g_finalize<GOP>(acc[i], deg);
             }
         }
     }
@@ -170,20 +198,28 @@ __global__ void __launch_bounds__(256) k_vertex_el(GraphArgs g, OpArgs op, int G
 cudaError_t launch_vertex_el(int kedge, int gather, const GraphArgs &g, const OpArgs &op, const LaunchCfg &c,
                              cudaStream_t s) {
     const int nc = (int)cdiv(op.W, c.vec);
-    const int64_t warps = cdiv(g.V, c.G);
-    if (warps == 0) return cudaSuccess;
-    const int64_t grid = cdiv(warps * 32, 256);
-#define UG_EL(NCV)                                                                                       \
+    const int64_t segs = cdiv(g.V, c.G);
+    if (segs == 0) return cudaSuccess;
+    const int64_t grid = cdiv(segs * c.L, 256);
+#define UG_EL(NCV, PV)                                                                                    \
     UG_DISPATCH_KE(kedge, KE,                                                                            \
-        UG_DISPATCH_RED(gather, GOP, k_vertex_el<KE, GOP, VEC, NCV><<<(unsigned)grid, 256, 0, s>>>(g, op, c.G)))
+        UG_DISPATCH_RED(gather, GOP,                                                                     \
+            k_vertex_el<KE, GOP, VEC, NCV, PV><<<(unsigned)grid, 256, 0, s>>>(g, op, c.G)))
+#define UG_EL_P(NCV)                                                                                     \
+    switch (c.L) {                                                                                       \
+    case 8: UG_EL(NCV, 8); break;                                                                        \
+    case 16: UG_EL(NCV, 16); break;                                                                      \
+    default: UG_EL(NCV, 32); break;                                                                      \
+    }
     UG_DISPATCH_VEC(c.vec, VEC, {
         switch (nc) {
-        case 1: UG_EL(1); break;
-        case 2: UG_EL(2); break;
-        case 3: case 4: UG_EL(4); break;
-        default: UG_EL(8); break;
+        case 1: UG_EL_P(1); break;
+        case 2: UG_EL_P(2); break;
+        case 3: case 4: UG_EL_P(4); break;
+        default: UG_EL_P(8); break;
         }
     });
+#undef UG_EL_P
 #undef UG_EL
     return cudaGetLastError();
 }

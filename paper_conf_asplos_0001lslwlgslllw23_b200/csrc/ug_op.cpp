@@ -167,15 +167,19 @@ ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, La
     }
     if (s.flags & UG_SCHED_EDGELANES) {
         // lanes over a row's in-edges (k_vertex_el): WV aggregation of an elementwise message, narrow W
-        if (c.strategy != UG_WV || lw.dot || lw.to_edges)
-            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "_E1: WV aggregation (or SV message creation) of an elementwise message only");
+        if ((c.strategy != UG_WV && c.strategy != UG_TV) || lw.dot || lw.to_edges)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "_E1: WV / TV aggregation (or SV message creation) of an elementwise message only");
+        // lanes per row: WV a whole warp (T must be 1); TV T in {8, 16} lanes, 32 / T rows per warp
+        const int T = s.tile > 0 ? s.tile : (c.strategy == UG_WV ? 1 : 0);
+        if (c.strategy == UG_WV ? T != 1 : (T != 8 && T != 16))
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "_E1: WV takes T1, TV takes T8 or T16 lanes per row");
         c.vec = s.vec ? s.vec : lw.max_vec;
         if (c.vec > lw.max_vec) return set_error(UG_ERR_ALIGNMENT, "forced vec wider than the operand layout allows");
         if ((lw.args.W + c.vec - 1) / c.vec > 8)
             return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "_E1: at most 8 feature vectors per row (W <= 8 * vec)");
         c.edgelanes = true;
         c.G = s.group > 0 ? s.group : 1;
-        c.L = 32;
+        c.L = c.strategy == UG_WV ? 32 : T;
         c.block = 256;
         *cfg = c;
         return UG_OK;

@@ -10,6 +10,6 @@ while [ $# -ge 2 ]; do
   NAME=$1; FLAGS=$2; shift 2
   touch $CS/*.cu; make -j16 EXTRA="$FLAGS" > gpurun_out/ab_build_$T-$NAME.log 2>&1 || { echo "build $NAME failed"; tail -5 gpurun_out/ab_build_$T-$NAME.log; continue; }
   echo "== $NAME ($FLAGS)"
-  timeout 900 python scripts/ab_sched.py --tag $T-$NAME --cases $CASES 2>&1 | grep '^{'
+  timeout 900 python scripts/ab_sched.py --tag $T-$NAME --reps ${AB_REPS:-20} --cases $CASES 2>&1 | grep '^{'
 done
 touch $CS/*.cu; make -j16 > /dev/null 2>&1

@@ -54,6 +54,7 @@ def candidates(cls, F, E, quick=False):
         c += [f"WV_G{g}_T1" for g in (1, 2, 8)]
         if cls != "dot_agg" and F <= 32:
             c += [f"WV_G{g}_T1_E1" for g in (1, 4)]       # lanes over in-edges (narrow F)
+            c += [f"TV_G1_T{t}_E1" for t in (8, 16)]       # 32 / t rows per warp, t edge lanes each
         c += [f"TE_G{g}_T{t}" for g in (1, 8, 32) for t in Ts if t >= 4]
         c += [f"WE_G{g}_T1" for g in (4, 32, 128)]
         vec = 4 if F % 4 == 0 else (2 if F % 2 == 0 else 1)
@@ -104,8 +105,13 @@ def time_schedule(g, kw, eo, go, sched, reps):
         ug.op_run(g, eo, go, schedule=sched, **kw)
         ev[2 * i + 1].record()
     torch.cuda.synchronize()
-    ts = [ev[2 * i].elapsed_time(ev[2 * i + 1]) for i in range(reps)]
-    return statistics.median(ts), None
+    ts = sorted(ev[2 * i].elapsed_time(ev[2 * i + 1]) for i in range(reps))
+    # interquartile mean: the event clock ticks in ~1.02 us steps, so on launch-bound graphs
+    # (C1 / C2) the median snaps to a tick; the middle half's mean dithers through it and still
+    # ignores outliers (equal to the median for the ms-scale ops)
+    q = len(ts) // 4
+    mid = ts[q:len(ts) - q] if len(ts) >= 4 else ts
+    return statistics.fmean(mid), None
 
 
 def logical_bytes(V, E, F, H, eo, go, a, b, c, wa, wb):

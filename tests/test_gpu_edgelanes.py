@@ -1,4 +1,5 @@
-"""GPU parity of the edge-lanes warp-vertex schedule ("WV_..._E1", k_vertex_el): every
+"""GPU parity of the edge-lanes vertex schedules ("WV_Gg_T1_E1": a warp per row, "TV_Gg_Tt_E1": t in
+{8, 16} lanes per row, 32 / t rows per warp; k_vertex_el): every
 aggregation op (all 32 message functions except dot x 4 reducers) in float mode (1e-5 * sum|terms|)
 and integer mode (bit-exact), widths 1..8 feature vectors, on an unsorted skewed multigraph
 (edge-id indirection, a hub row wider than the warp, zero in-degree rows)."""
@@ -31,7 +32,7 @@ def test_edgelanes_all_aggregations(graph, op, mode):
     for (F, H, ew) in ((20, 1, 1), (12, 3, 3), (32, 1, 32), (4, 1, 1)):
         A, B = operand_arrays(op, V, E, F, H, seed=F, mode=mode, edge_width=ew)
         ref, bound = run_oracle(op, V, src, dst, A, B, F, H)
-        for sch in ("WV_G1_T1_E1", "WV_G4_T1_E1"):
+        for sch in ("WV_G1_T1_E1", "WV_G4_T1_E1", "TV_G1_T8_E1", "TV_G3_T16_E1"):
             got = run_gpu(ug, g, op, A, B, V, E, F, H, schedule=sch)
             assert_parity(op, got, ref, bound, mode == "int", what=f"{name(op)} {sch} F={F} H={H}")
 
@@ -47,9 +48,10 @@ def test_edgelanes_rejects(graph):
     with pytest.raises(ug.UgError):      # message creation
         ug.op_run(g, "copy_lhs", "assign", A=X[:, :8], a_type="u", C=M, c_type="e", F=8,
                   schedule="WV_G1_T1_E1")
-    with pytest.raises(ug.UgError):      # not WV
-        ug.op_run(g, "copy_lhs", "sum", A=X[:, :8], a_type="u", C=Y[:, :8], c_type="v", F=8,
-                  schedule="TV_G1_T1_E1")
+    for bad in ("TV_G1_T1_E1", "TV_G1_T4_E1", "WV_G1_T2_E1", "BV_G1_E1"):   # lanes per row: WV 32, TV 8 / 16
+        with pytest.raises(ug.UgError):
+            ug.op_run(g, "copy_lhs", "sum", A=X[:, :8], a_type="u", C=Y[:, :8], c_type="v", F=8,
+                      schedule=bad)
     assert ug.format_schedule(ug.parse_schedule("WV_G4_T1_E1")) == "WV_G4_T1_E1"
 
 
