@@ -49,7 +49,9 @@ __device__ __forceinline__ float warp_sum8_transposed(float (&v)[8], int lane) {
 #define UG_DOTT_MINB 6
 #endif
 
-template <int VEC>
+// O32: every row of P is addressable with a 32-bit element offset (V_src * ld < 2^32): the gather
+// address is one IMAD + IMAD.WIDE from the column index, as in the SV aggregation kernel
+template <int VEC, bool O32>
 __global__ void __launch_bounds__(256, UG_DOTT_MINB) k_dott(GraphArgs g, OpArgs op, bool a_is_src,
                                                             const int4 *__restrict__ chunks, int n_chunks,
                                                             int tiles_per_head, float *__restrict__ out,
@@ -76,7 +78,7 @@ __global__ void __launch_bounds__(256, UG_DOTT_MINB) k_dott(GraphArgs g, OpArgs 
 #pragma unroll
         for (int i = 0; i < VEC; ++i) q[i] = i < nval ? Q.p[v * Q.ld + f + i] : 0.0f;
     const float *__restrict__ Pb = P.p + f;
-    const uint32_t ldp = (uint32_t)P.ld;
+    const uint32_t ldp = (uint32_t)P.ld, fo32 = (uint32_t)f;
     float *dst = out + (int64_t)t * tile_stride + o;
     const int k1 = ch.z;
     // a batch: 8 column indices, then 8 row gathers (UG_DOTT_PIPE=1 issues the next batch's before
@@ -94,7 +96,10 @@ __global__ void __launch_bounds__(256, UG_DOTT_MINB) k_dott(GraphArgs g, OpArgs 
             for (int i = 0; i < 8; ++i) s_pf[i] = (uint32_t)ldg_i32_hint(g.col + min(ch.y + i, last), stream);
         }
     }
-    auto load_batch = [&](int k, float (&x)[8][VEC]) {
+    // MASK: only a head's last column tile can hold inactive lanes or a ragged tail; full tiles
+    // (every lane nval == VEC, warp-uniform) skip the 8 x VEC selects per batch (UG_DOTT_FULL)
+    auto load_batch = [&](auto mask_tag, int k, float (&x)[8][VEC]) {
+        constexpr bool MASK = decltype(mask_tag)::value;
         uint32_t s[8];
         if constexpr (UG_DOTT_PF) {
 #pragma unroll
@@ -111,9 +116,12 @@ __global__ void __launch_bounds__(256, UG_DOTT_MINB) k_dott(GraphArgs g, OpArgs 
             // branch-free: every lane loads a full vector from a valid address (an inactive lane
             // its head's first columns; a ragged tail reads into the packed row's padding) and
             // zeroes the elements outside the head by select
-            ldg_vec_hint<VEC>(Pb + s[i] * ldp, x[i], keep);
+            if constexpr (O32) ldg_vec_hint<VEC>(P.p + (s[i] * ldp + fo32), x[i], keep);
+            else ldg_vec_hint<VEC>(Pb + s[i] * ldp, x[i], keep);
+            if constexpr (MASK) {
 #pragma unroll
-            for (int j = 0; j < VEC; ++j) x[i][j] = j < nval ? x[i][j] : 0.0f;
+                for (int j = 0; j < VEC; ++j) x[i][j] = j < nval ? x[i][j] : 0.0f;
+            }
         }
     };
     float xa[8][VEC];
@@ -137,22 +145,33 @@ __global__ void __launch_bounds__(256, UG_DOTT_MINB) k_dott(GraphArgs g, OpArgs 
 #ifndef UG_DOTT_PIPE
 #define UG_DOTT_PIPE 0
 #endif
+#ifndef UG_DOTT_FULL
+#define UG_DOTT_FULL 1
+#endif
+    using masked = std::true_type;
     if constexpr (!UG_DOTT_PIPE) {
         // one batch in flight per warp: a second (software-pipelined) batch measured slower at every
         // vector width (registers: 64 at VEC 2, spills at VEC 4; profiles/r2/ab_r2l.jsonl)
-        for (; k < k1; k += 8) {
-            load_batch(k, xa);
-            reduce_store(k, xa);
+        if (UG_DOTT_FULL && __all_sync(0xffffffffu, nval == VEC)) {
+            for (; k < k1; k += 8) {
+                load_batch(std::false_type{}, k, xa);
+                reduce_store(k, xa);
+            }
+        } else {
+            for (; k < k1; k += 8) {
+                load_batch(masked{}, k, xa);
+                reduce_store(k, xa);
+            }
         }
     } else {
         float xb[8][VEC];
-        if (k < k1) load_batch(k, xa);
+        if (k < k1) load_batch(masked{}, k, xa);
         while (k < k1) {
-            if (k + 8 < k1) load_batch(k + 8, xb);
+            if (k + 8 < k1) load_batch(masked{}, k + 8, xb);
             reduce_store(k, xa);
             k += 8;
             if (k >= k1) break;
-            if (k + 8 < k1) load_batch(k + 8, xa);
+            if (k + 8 < k1) load_batch(masked{}, k + 8, xa);
             reduce_store(k, xb);
             k += 8;
         }
@@ -171,6 +190,9 @@ __global__ void k_dott_fix(const float *__restrict__ part, int64_t E, int H, int
     C[e * c_ld + o] = s;
 }
 
+#ifndef UG_DOTT_O32
+#define UG_DOTT_O32 1
+#endif
 int dott_tiles(const OpArgs &op, int vec) { return (int)cdiv(op.D, 32 * vec); }
 
 // Message creation into C (c_ld) -- or, when tiles > 1, partials into `part` ([tiles][E][H]) and
@@ -189,9 +211,16 @@ cudaError_t launch_dott(const GraphArgs &g, const OpArgs &op, bool a_is_src, int
     const int64_t dld = direct ? c_ld : op.H;
     const int64_t tstride = (int64_t)g.E * op.H;
     if (ev_begin) cudaEventRecord(ev_begin, s);
-    UG_DISPATCH_VEC(vec, VEC,
-        k_dott<VEC><<<(unsigned)grid, 256, 0, s>>>(g, op, a_is_src, chunks, (int)plan.n_chunks, th, dst, dld,
-                                                   tstride));
+    const Operand &P = a_is_src ? op.A : op.B;
+    const bool o32 = (uint64_t)g.V_src * (uint64_t)P.ld < (1ull << 32) && UG_DOTT_O32;
+    UG_DISPATCH_VEC(vec, VEC, {
+        if (o32)
+            k_dott<VEC, true><<<(unsigned)grid, 256, 0, s>>>(g, op, a_is_src, chunks, (int)plan.n_chunks, th, dst,
+                                                             dld, tstride);
+        else
+            k_dott<VEC, false><<<(unsigned)grid, 256, 0, s>>>(g, op, a_is_src, chunks, (int)plan.n_chunks, th, dst,
+                                                              dld, tstride);
+    });
     if (ev_end) cudaEventRecord(ev_end, s);
     cudaError_t err = cudaGetLastError();
     if (err != cudaSuccess || direct) return err;

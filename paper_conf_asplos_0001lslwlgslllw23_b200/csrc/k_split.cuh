@@ -22,7 +22,8 @@ namespace ug {
 
 // Inner in-edge loop of the SV fast path.  BM: 0 no B operand, 1 B is Dst_V (constant over
 // the row: loaded once), 2 / 3 B is an Edge tensor (row = CSR position) with per-head broadcast
-// / full width, 4 / 5 B is Src_V with broadcast / full width.  All offsets are 32-bit (the
+// / full width, 4 / 5 B is Src_V with broadcast / full width, 6 / 7 B is a per-edge scalar stored
+// contiguously (GCN's edge weight; 7 = the same loop at 8 CTAs / SM).  All offsets are 32-bit (the
 // host checks rows * ld < 2^32).  The last, partial group of UF edges is predicated (its
 // missing slots re-read the row's last edge, an L1 hit, and are not combined), so short rows
 // never fall into a serial one-edge-at-a-time tail.  
@@ -38,7 +39,7 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
 #define UG_BM6_UF UG_BM2_UF
 #endif
     constexpr int UF = BM == 0 || BM == 1 ? (VEC == 4 ? 8 : 16)
-                     : (BM == 6 && KE != K_DIV) ? UG_BM6_UF
+                     : (BM >= 6 && KE != K_DIV) ? UG_BM6_UF
                      : (BM == 2 && KE != K_DIV) ? UG_BM2_UF : (VEC == 4 ? 4 : 8) / (KE == K_DIV ? 2 : 1);
     const float *__restrict__ Ab = op.A.p;          // warp-uniform base
     const uint64_t keep = l2_policy_evict_last();     // this tile's X column slab
@@ -47,7 +48,7 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
     // BM 6: a per-edge scalar stored contiguously (ld 1, column 0) -- the weight of position k is
     // B.p[k], addressed like col_idx (one pointer, immediate offsets; no per-edge IMAD / offset
     // registers)
-    const uint32_t ldb = BM == 6 ? 1u : (uint32_t)op.B.ld, cbo = BM == 6 ? 0u : (uint32_t)cb;
+    const uint32_t ldb = BM >= 6 ? 1u : (uint32_t)op.B.ld, cbo = BM >= 6 ? 0u : (uint32_t)cb;
     constexpr bool bfull = BM == 3 || BM == 5;
     float bconst[VEC];
     if constexpr (BM == 1) fetch<VEC>(op.B, v, cb, bconst);
@@ -92,7 +93,7 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
 #endif
         // UG_MUL_FMA: a per-edge scalar weight folded into the sum by FMA (the message is then not
         // rounded on its own -- within R11's bound, exact in integer mode); A/B switch
-        constexpr bool FMA_W = UG_MUL_FMA && (BM == 2 || BM == 6) && KE == K_MUL && (GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN);
+        constexpr bool FMA_W = UG_MUL_FMA && (BM == 2 || BM >= 6) && KE == K_MUL && (GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN);
         if constexpr (FMA_W) {
             float wq[UF];
 #pragma unroll
@@ -113,10 +114,10 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
 #pragma unroll
                     for (int i = 0; i < VEC; ++i) b[i] = bconst[i];
                 } else {
-                    const uint32_t row = (BM == 2 || BM == 3 || BM == 6) ? (uint32_t)(PRED ? min(k + q, kl) : k + q) : s[q];
+                    const uint32_t row = (BM == 2 || BM == 3 || BM >= 6) ? (uint32_t)(PRED ? min(k + q, kl) : k + q) : s[q];
                     // BM 6: 64-bit position arithmetic, so B.p + k becomes one pointer with
                     // immediate offsets (as for col_idx) instead of a 32-bit IMAD per edge
-                    const float *bp = BM == 6 ? op.B.p + (PRED ? min(k + q, kl) : k + q) : op.B.p + (row * ldb + cbo);
+                    const float *bp = BM >= 6 ? op.B.p + (PRED ? min(k + q, kl) : k + q) : op.B.p + (row * ldb + cbo);
                     if constexpr (bfull) {
                         ldg_vec_hint<VEC>(bp, b, BM == 3 ? stream : keep);
                     } else {
@@ -161,7 +162,7 @@ __device__ __forceinline__ void split_fast_assign(const GraphArgs &g, const OpAr
     const float *__restrict__ Ab = op.A.p;
     const uint64_t keep = l2_policy_evict_last(), stream = l2_policy_evict_first();
     const uint32_t lda = (uint32_t)op.A.ld, fo = (uint32_t)f;
-    const uint32_t ldb = BM == 6 ? 1u : (uint32_t)op.B.ld, cbo = BM == 6 ? 0u : (uint32_t)cb;
+    const uint32_t ldb = BM >= 6 ? 1u : (uint32_t)op.B.ld, cbo = BM >= 6 ? 0u : (uint32_t)cb;
     constexpr bool bfull = BM == 3 || BM == 5;
     const int nout = op.W - f;
     const bool full_vec = nout >= VEC && op.c_vec >= VEC;
@@ -175,7 +176,7 @@ __device__ __forceinline__ void split_fast_assign(const GraphArgs &g, const OpAr
 #pragma unroll
                 for (int i = 0; i < VEC; ++i) b[i] = bconst[i];
             } else {
-                const uint32_t row = (BM == 2 || BM == 3 || BM == 6) ? (uint32_t)kk : sq;
+                const uint32_t row = (BM == 2 || BM == 3 || BM >= 6) ? (uint32_t)kk : sq;
                 const float *bp = op.B.p + (row * ldb + cbo);
                 if constexpr (bfull) {
                     ldg_vec_hint<VEC>(bp, b, BM == 3 ? stream : keep);
@@ -223,6 +224,12 @@ __device__ __forceinline__ void split_fast_assign(const GraphArgs &g, const OpAr
 // BM = 6 (a per-edge scalar stored contiguously): its addressing frees the per-edge offset registers
 #ifndef UG_BM6_SUM_MINB
 #define UG_BM6_SUM_MINB 6
+#endif
+// BM = 7: the BM 6 loop at 8 CTAs / SM (32 registers) for sum / mean on short-chunk graphs with
+// many waves -- C3 u_mul_e_sum F = 128 268.5 -> 252.2 us, C4 92.4 -> 86.3 us, but C5 (long chunks)
+// 19.5 -> 21.3 ms and C2 (one wave) 13.6 -> 15.6 us (profiles/r2/ab_r2i.jsonl); chosen at launch
+#ifndef UG_BM7_MINB
+#define UG_BM7_MINB 8
 #endif
 #ifndef UG_BM0_MINB
 #define UG_BM0_MINB 8
@@ -370,7 +377,7 @@ template <int KE, int GOP, int VEC, int BM, bool MERGE>
 #ifndef UG_ASSIGN_MINB
 #define UG_ASSIGN_MINB 6
 #endif
-__global__ void __launch_bounds__(256, (UG_ASSIGN_MINB > 0 && GOP == UG_GATHER_ASSIGN) ? UG_ASSIGN_MINB : (BM == 0) ? UG_BM0_MINB : (BM == 6 && (GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN) && KE != K_DIV) ? UG_BM6_SUM_MINB : ((BM == 2 || BM == 6) ? ((GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN) && KE != K_DIV ? UG_BM2_SUM_MINB : UG_BM2_MINB) : (BM > 0 ? (VEC == 4 ? 5 : 6) : 4))) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
+__global__ void __launch_bounds__(256, (UG_ASSIGN_MINB > 0 && GOP == UG_GATHER_ASSIGN) ? UG_ASSIGN_MINB : (BM == 0) ? UG_BM0_MINB : (BM == 7) ? UG_BM7_MINB : (BM == 6 && (GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN) && KE != K_DIV) ? UG_BM6_SUM_MINB : ((BM == 2 || BM == 6) ? ((GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN) && KE != K_DIV ? UG_BM2_SUM_MINB : UG_BM2_MINB) : (BM > 0 ? (VEC == 4 ? 5 : 6) : 4))) k_split(GraphArgs g, OpArgs op, const int4 *__restrict__ chunks,
                                                int64_t n_chunks, int L_log2, int ftile, int n_tiles,
                                                float *__restrict__ scratch, int64_t sld,
                                                const int4 *__restrict__ split, const int32_t *__restrict__ slot_row,
@@ -424,6 +431,9 @@ __global__ void k_split_fix(GraphArgs g, OpArgs op, const int4 *__restrict__ spl
 #ifndef UG_SV_BM6
 #define UG_SV_BM6 1
 #endif
+#ifndef UG_SV_BM7
+#define UG_SV_BM7 1
+#endif
 // Launch of one edge_op's SV instances (explicitly instantiated per KE in k_split*.cu).
 template <int KE>
 cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, const LaunchCfg &c,
@@ -453,6 +463,10 @@ cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, co
     const int bm = !fast ? -1 : KE == K_COPY ? 0
                  : op.B.type == UG_T_DST_V ? 1
                  : op.B.type == UG_T_EDGE ? (op.B.div == op.W && op.B.ld == 1 && UG_SV_BM6 ? 6 : 2 + bfl) : 4 + bfl;
+    // occupancy instance of BM 6 (see UG_BM7_MINB): short chunks (< 32 in-edges on average) and a
+    // grid of at least four waves at 8 CTAs / SM
+    const bool short_chunks = plan.n_chunks > 0 && g.E < 32 * plan.n_chunks;
+    const int bm_launch = (bm == 6 && UG_SV_BM7 && short_chunks && threads >= (int64_t)4 * 148 * 2048) ? 7 : bm;
 #define UG_SV_LAUNCH(BMV)                                                                                    \
     do {                                                                                                     \
         if constexpr (GOP != UG_GATHER_ASSIGN) {                                                             \
@@ -472,13 +486,17 @@ cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, co
             if constexpr (KE == K_COPY) {
                 if (bm == 0) UG_SV_LAUNCH(0); else UG_SV_LAUNCH(-1);
             } else {
-                switch (bm) {
+                switch (bm_launch) {
                 case 1: UG_SV_LAUNCH(1); break;
                 case 2: UG_SV_LAUNCH(2); break;
                 case 3: UG_SV_LAUNCH(3); break;
                 case 4: UG_SV_LAUNCH(4); break;
                 case 5: UG_SV_LAUNCH(5); break;
                 case 6: UG_SV_LAUNCH(6); break;
+                case 7:
+                    if constexpr ((GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN) && KE != K_DIV) UG_SV_LAUNCH(7);
+                    else UG_SV_LAUNCH(6);
+                    break;
                 default: UG_SV_LAUNCH(-1); break;
                 }
             }

@@ -10,7 +10,7 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 60 --cs
 timeout 1200 ncu --set full --clock-control none --import-source on -k regex:'^k_split$' -s 3 -c 1 -o gpurun_out/prof_k_split_$T python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-e2e --no-secondary > gpurun_out/ncu_$T.log 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,lts__t_sector_hit_rate.pct,lts__t_sectors_srcunit_tex_op_read.sum --clock-control none -k regex:'^k_' --csv --log-file gpurun_out/ncu_per_op_$T.csv python scripts/ncu_per_op.py run gpurun_out/ncu_per_op_order_$T.json > gpurun_out/ncu_per_op_$T.log 2>&1; tail -1 gpurun_out/ncu_per_op_$T.log
 UG_DIST_BACKEND=gloo timeout 1200 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 5 --warmup 3 > gpurun_out/bench_dry2_$T.log 2>&1; tail -c 300 gpurun_out/bench_dry2_$T.log
-timeout 1500 python scripts/sweep.py --configs C1 C2 C3 C4 C5 --out gpurun_out/sweep_$T.jsonl 2>&1 | grep -v Warn | tail -3
+timeout 2400 python scripts/sweep.py --configs C1 C2 C3 C4 C5 --reps 10 --out gpurun_out/sweep_$T.jsonl 2>&1 | grep -v Warn | tail -3
 for TOOL in memcheck racecheck synccheck; do
   timeout 1200 compute-sanitizer --tool $TOOL python scripts/sanitize.py > gpurun_out/sanitize_${TOOL}_$T.log 2>&1
   tail -2 gpurun_out/sanitize_${TOOL}_$T.log
