@@ -21,7 +21,9 @@ namespace ug {
 #define UG_DOTSV_MINB 4   // resident CTAs per SM the register budget is sized for
 #endif
 
-template <int GOP, int VEC, int NJ>
+// O32: every row of P is addressable with a 32-bit element offset (V_src * ld < 2^32): a gather
+// address is one IMAD + IMAD.WIDE from the column index instead of 64-bit multiply / LEA pairs
+template <int GOP, int VEC, int NJ, bool O32>
 __global__ void __launch_bounds__(256, UG_DOTSV_MINB) k_dotsv(GraphArgs g, OpArgs op, bool a_is_src, const int4 *__restrict__ chunks,
                                                   int64_t n_chunks, int L_log2, int w_log2,
                                                   float *__restrict__ scratch, int64_t sld) {
@@ -53,6 +55,12 @@ __global__ void __launch_bounds__(256, UG_DOTSV_MINB) k_dotsv(GraphArgs g, OpArg
     const float *__restrict__ Pb = P.p + f0;
     const int jstride = w * VEC;
     const int64_t ldp = P.ld;
+    const uint32_t ldp32 = (uint32_t)P.ld, f032 = (uint32_t)f0;
+    // gather of chunk j of source row src
+    auto gather = [&](int64_t src, int j, float (&r)[VEC]) {
+        if constexpr (O32) ldg_vec_hint<VEC>(P.p + ((uint32_t)src * ldp32 + f032 + (uint32_t)(j * jstride)), r, keep);
+        else ldg_vec_hint<VEC>(Pb + src * ldp + j * jstride, r, keep);
+    };
 
     float acc = g_init<GOP>();
     auto edge_msg = [&](const float (&p)[NJ][VEC]) {
@@ -103,7 +111,7 @@ __global__ void __launch_bounds__(256, UG_DOTSV_MINB) k_dotsv(GraphArgs g, OpArg
         for (int e = 0; e < UE; ++e) {
 #pragma unroll
             for (int j = 0; j < NJ; ++j) {
-                if (active) ldg_vec_hint<VEC>(Pb + s[e] * ldp + j * jstride, p[e][j], keep);
+                if (active) gather(s[e], j, p[e][j]);
                 else
 #pragma unroll
                     for (int i = 0; i < VEC; ++i) p[e][j][i] = 0.0f;
@@ -120,7 +128,7 @@ __global__ void __launch_bounds__(256, UG_DOTSV_MINB) k_dotsv(GraphArgs g, OpArg
         if (k + 1 < k1) s_next = ldg_i32_hint(g.col + k + 1, stream);
 #pragma unroll
         for (int j = 0; j < NJ; ++j) {
-            if (active) ldg_vec_hint<VEC>(Pb + s * ldp + j * jstride, p[j], keep);
+            if (active) gather(s, j, p[j]);
             else
 #pragma unroll
                 for (int i = 0; i < VEC; ++i) p[j][i] = 0.0f;
@@ -143,6 +151,9 @@ __global__ void __launch_bounds__(256, UG_DOTSV_MINB) k_dotsv(GraphArgs g, OpArg
 // (fewer butterfly steps per edge: measured on C4 F=128, 8 lanes x 16 features 98 us against
 // 32 lanes x 4 features 167 us).  Returns NJ, or 0 when the op does not fit (the caller then
 // uses the generic dot kernel).
+#ifndef UG_DOTSV_O32
+#define UG_DOTSV_O32 1
+#endif
 int dotsv_nj(const OpArgs &op, int vec, int *L, int *w) {
     for (int nj : {4, 2, 1}) {
         const int per = nj * vec;
@@ -172,9 +183,19 @@ cudaError_t launch_dotsv(int gather, const GraphArgs &g, const OpArgs &op, bool 
     const int64_t sld = cdiv(op.W, 4) * 4;
     const int4 *chunks = reinterpret_cast<const int4 *>(plan.d_chunk);
     if (ev_begin) cudaEventRecord(ev_begin, s);
+    const Operand &P = a_is_src ? op.A : op.B;
+    const bool o32 = (uint64_t)g.V_src * (uint64_t)P.ld < (1ull << 32) && UG_DOTSV_O32;
 #define UG_DOTSV(NJV)                                                                                     \
-    k_dotsv<GOP, VEC, NJV><<<(unsigned)grid, block, 0, s>>>(g, op, a_is_src, chunks, plan.n_chunks,      \
-                                                           ilog2(L), ilog2(w), scratch, sld)
+    do {                                                                                                  \
+        if (o32)                                                                                          \
+            k_dotsv<GOP, VEC, NJV, true><<<(unsigned)grid, block, 0, s>>>(g, op, a_is_src, chunks,       \
+                                                                          plan.n_chunks, ilog2(L),        \
+                                                                          ilog2(w), scratch, sld);        \
+        else                                                                                              \
+            k_dotsv<GOP, VEC, NJV, false><<<(unsigned)grid, block, 0, s>>>(g, op, a_is_src, chunks,      \
+                                                                           plan.n_chunks, ilog2(L),       \
+                                                                           ilog2(w), scratch, sld);       \
+    } while (0)
     UG_DISPATCH_VEC(vec, VEC,
         UG_DISPATCH_GOP(gather, GOP, {
             switch (nj) {

@@ -89,15 +89,19 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
 #pragma unroll
         for (int q = 0; q < UF; ++q) ldg_vec_hint<VEC>(Ab + (s[q] * lda + fo), m[q], keep);
 #ifndef UG_MUL_FMA
-#define UG_MUL_FMA 0
+#define UG_MUL_FMA 1
 #endif
-        // UG_MUL_FMA: a per-edge scalar weight folded into the sum by FMA (the message is then not
-        // rounded on its own -- within R11's bound, exact in integer mode); A/B switch
-        constexpr bool FMA_W = UG_MUL_FMA && (BM == 2 || BM >= 6) && KE == K_MUL && (GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN);
+        // UG_MUL_FMA: a per-edge scalar weight folded into the sum by FMA (the message x * w is then
+        // rounded together with the add, not on its own -- inside R11's 1e-5 * sum|terms| bound,
+        // exact in integer mode).  On with the contiguous-weight loops: C5 u_mul_e_sum 19.19 ->
+        // 18.71 ms, C3 F = 128 256.3 -> 254.2 us (profiles/r2/ab_r2l.jsonl; r2 with BM 2 it lost)
+        constexpr bool FMA_W = UG_MUL_FMA && BM >= 6 && KE == K_MUL && (GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN);
         if constexpr (FMA_W) {
             float wq[UF];
 #pragma unroll
-            for (int q = 0; q < UF; ++q) wq[q] = __ldg(op.B.p + ((uint32_t)(PRED ? min(k + q, kl) : k + q) * ldb + cbo));
+            for (int q = 0; q < UF; ++q)
+                wq[q] = BM >= 6 ? __ldg(op.B.p + (PRED ? min(k + q, kl) : k + q))
+                                : __ldg(op.B.p + ((uint32_t)(PRED ? min(k + q, kl) : k + q) * ldb + cbo));
 #pragma unroll
             for (int q = 0; q < UF; ++q) {
                 const bool ok = !PRED || k + q < k1;
@@ -347,7 +351,7 @@ __device__ __forceinline__ void split_merge(const GraphArgs &g, const OpArgs &op
     if (!last) return;
     fence_acq_rel_gpu();
     if (lane == 0) counters[(int64_t)r * n_tiles + tile] = 0;
-    if (f >= op.W) return;
+    if (f >= op.W || lane * VEC >= ftile) return;
     float acc[VEC];
 #pragma unroll
     for (int i = 0; i < VEC; ++i) acc[i] = g_init<GOP>();
@@ -388,15 +392,16 @@ __global__ void __launch_bounds__(256, (UG_ASSIGN_MINB > 0 && GOP == UG_GATHER_A
     if (u >= n_chunks * n_tiles) return;          // whole units only: a unit's L lanes leave together
     const int tile = unit_tile(u, n_chunks, n_tiles);
     const int f = tile * ftile + lane * VEC;
+    const bool lane_ok = lane * VEC < ftile;       // false only for the idle lanes of a non-pow2 tile
     if constexpr (!MERGE) {
         // split rows (if any) are combined by k_split_fix, a second launch
-        if (f >= op.W) return;
+        if (f >= op.W || !lane_ok) return;
         split_unit<KE, GOP, VEC, BM>(g, op, chunks[u - (int64_t)tile * n_chunks], f, scratch, sld);
     } else {
         // single-launch merge of split rows: the last-arriving chunk of a row combines them.  A
         // separate instance (launch-bound small graphs): the merge needs every lane of the unit
         // and re-derives its indices after the in-edge loop.
-        if (f < op.W) split_unit<KE, GOP, VEC, BM>(g, op, chunks[u - (int64_t)tile * n_chunks], f, scratch, sld);
+        if (f < op.W && lane_ok) split_unit<KE, GOP, VEC, BM>(g, op, chunks[u - (int64_t)tile * n_chunks], f, scratch, sld);
         split_merge<GOP, VEC>(g, op, chunks, n_chunks, L_log2, ftile, n_tiles, scratch, sld, split, slot_row,
                               counters);
     }
@@ -439,7 +444,8 @@ template <int KE>
 cudaError_t launch_split_ke(int gather, const GraphArgs &g, const OpArgs &op, const LaunchCfg &c,
                             const SplitPlan &plan, float *scratch, cudaStream_t s, cudaEvent_t ev_begin,
                             cudaEvent_t ev_end, int32_t *counters) {
-    const int L = c.ftile / c.vec;
+    int L = 1;
+    while (L * c.vec < c.ftile) L <<= 1;        // lanes past ftile / vec (a non-power-of-two tile) idle
     const int n_tiles = (int)cdiv(op.W, c.ftile);
     const int64_t threads = plan.n_chunks * n_tiles * (int64_t)L;
     if (threads == 0) return cudaSuccess;

@@ -268,9 +268,11 @@ ug_status resolve(const ug_graph *g, const Lowered &lw, const ug_schedule &s, La
     if (c.ftile < 0 || c.ftile % c.vec) return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "ftile must be a multiple of vec");
     if (c.strategy == UG_SV && !lw.dot) {
         if (c.ftile == 0) c.ftile = std::min(32, need) * c.vec;
-        const int L = c.ftile / c.vec;
-        if (!is_pow2(L) || L > 32)
-            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "SV needs ftile / vec a power of two <= 32");
+        // lanes per unit: ftile / vec rounded up to a power of two (lanes past ftile idle), so a
+        // column tile need not be a power-of-two width (e.g. F120: 30 float4 lanes of 32)
+        const int L = pow2ceil(c.ftile / c.vec);
+        if (c.ftile / c.vec > 32)
+            return set_error(UG_ERR_UNSUPPORTED_SCHEDULE, "SV needs ftile / vec <= 32");
         c.L = L;
     }
     if (c.strategy == UG_BE) c.L = std::min(32, need);

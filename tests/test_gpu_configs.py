@@ -109,7 +109,7 @@ def test_C3_schedule_sweep(sch):
 
 
 @pytest.mark.parametrize("sch", [None, "SV_G2048_F64", "SV_G1024_F32", "SV_G512_F64_P1", "SV_G512_F128_P1", "WV_G1_T1",
-                                 "BV_G1_B512"])
+                                 "BV_G1_B512", "SV_G512_F120_P1"])
 @pytest.mark.parametrize("gop", ["sum", "mean"])
 def test_C5_headline(sch, gop):
     """C5 copy_u_sum / copy_u_mean at F=602 (the bench workload) on several schedules."""
@@ -125,7 +125,7 @@ def test_C5_padded_and_cross_schedule_integer():
     Xp = to_dev(X, ld=608)
     outs = []
     for sch, XX in (("SV_G2048_F64", Xd), ("WV_G1_T1", Xd), ("BV_G1_B256", Xd), ("SV_G2048_F64", Xp),
-                    ("SV_G2048_F64_P1", Xd), ("SV_G512_F128_P1", Xd)):
+                    ("SV_G2048_F64_P1", Xd), ("SV_G512_F128_P1", Xd), ("SV_G512_F120_P1", Xd)):
         C = torch.empty(d["V"], 602, device="cuda")
         ug.op_run(d["g"], "copy_lhs", "sum", A=XX, a_type="u", C=C, c_type="v", schedule=sch)
         outs.append(C)

@@ -166,3 +166,29 @@ def test_message_creation_sv_fast_path(mode):
             for sch in ("SV_G7", "SV_G64_F8", "SV_G16_P1", "SV_G32_F64"):
                 got = run_gpu(ug, g, op, A, B, V, E, F, H, schedule=sch)
                 assert_parity(op, got, ref, bound, mode == "int", what=f"{name(op)} {sch} F={F}")
+
+
+@pytest.mark.parametrize("mode", ["float", "int"])
+@pytest.mark.parametrize("kind", ["sorted", "unsorted"])
+def test_sv_non_power_of_two_tiles(mode, kind):
+    """SV column tiles whose width is not a power of two lanes (F12 / F24 / F40 at float4: 3, 6, 10
+    lanes of a 4 / 8 / 16-lane unit, the rest idle) on every aggregation op: the fast path with
+    each B addressing mode (sorted graph, incl. the contiguous edge weight of BM 6) and the generic
+    one (unsorted: eid), the single-launch merge of split rows (small operator) included."""
+    V, E = 300, 1500
+    src, dst = ugdata.random_multigraph(V, E, 79, zero_in_frac=0.15)
+    hub = np.arange(0, 140, dtype=np.int32)
+    src = np.concatenate([src, hub]).astype(np.int32)
+    dst = np.concatenate([dst, np.full(140, 11, np.int32)]).astype(np.int32)
+    if kind == "sorted":
+        order = np.argsort(dst, kind="stable")
+        src, dst = src[order], dst[order]
+    E = len(src)
+    g = ug.Graph(V, src, dst)
+    for op in [o for o in all_ops() if o[4] == "v" and o[0] != "dot"]:
+        for (F, H, ew) in ((20, 1, 1), (24, 2, 2)):
+            A, B = operand_arrays(op, V, E, F, H, seed=F + 5, mode=mode, edge_width=ew)
+            ref, bound = run_oracle(op, V, src, dst, A, B, F, H)
+            for sch in ("SV_G7_F12", "SV_G64_F24_P1", "SV_G16_F40"):
+                got = run_gpu(ug, g, op, A, B, V, E, F, H, schedule=sch)
+                assert_parity(op, got, ref, bound, mode == "int", what=f"{name(op)} {sch} F={F} {kind}")
