@@ -195,9 +195,104 @@ __global__ void __launch_bounds__(256) k_vertex_el(GraphArgs g, OpArgs op, int G
     }
 }
 
+// Segmented edge lanes ("WV_Gg_T1_E1", g in {2, 4, 8}, round 2): the warp's g consecutive rows
+// share its 32 lanes -- their in-edges are the consecutive CSR positions [row_ptr[v0],
+// row_ptr[v0 + g]), lane l takes positions base + l, base + l + 32, ... and accumulates each
+// message into the partial of its row (found from the g + 1 row boundaries, loaded once per warp).
+// A hub row no longer serialises over one sub-warp's lanes (TV_G1_T8_E1: ceil(d / 16) steps) and
+// light rows no longer leave most of a warp idle (WV_G1_T1_E1).  The g x N partials are combined
+// by one transposed butterfly (g N <= 32 values: g N - 1 shuffles), which leaves value j = (row,
+// feature) in lanes j * (32 / g N) ...; owner computes, one launch.
+template <int KE, int GOP, int VEC, int NC, int G>
+__global__ void __launch_bounds__(256) k_vertex_seg(GraphArgs g, OpArgs op) {
+    constexpr int N = NC * VEC;                       // values per row (a power of two)
+    constexpr int NT = G * N;                         // values per warp, <= 32
+    static_assert(NT <= 32, "segmented edge lanes: G * N <= 32");
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    const int64_t v0 = warp * G;
+    if (v0 >= g.V) return;                            // whole warps leave together
+    int64_t b[G + 1];                                 // row boundaries (warp-uniform loads)
+#pragma unroll
+    for (int r = 0; r <= G; ++r) b[r] = (int64_t)g.row_ptr[min(v0 + r, g.V)] - g.rp_base;
+    int64_t ca[NC], cb[NC];
+#pragma unroll
+    for (int j = 0; j < NC; ++j) {
+        ca[j] = op_col(op.A, min(j * VEC, op.W - 1));
+        cb[j] = op_col(op.B, min(j * VEC, op.W - 1));
+    }
+    float acc[NT];
+#pragma unroll
+    for (int j = 0; j < NT; ++j) acc[j] = g_init<GOP>();
+    auto add_edge = [&](int64_t k) {
+        int r = 0;                                    // local row of position k
+#pragma unroll
+        for (int i = 1; i < G; ++i) r += k >= b[i];
+        const int64_t v = v0 + r;
+        const int64_t src = g.col[k];
+        const int64_t e = g.eid ? (int64_t)g.eid[k] : k;
+        const int64_t ra = op_row(op.A.type, src, v, e), rb = op_row(op.B.type, src, v, e);
+#pragma unroll
+        for (int j = 0; j < NC; ++j) {
+            if (j * VEC < op.W) {
+                float m[VEC];
+                message<KE, VEC>(op, ra, ca[j], rb, cb[j], m);
+#pragma unroll
+                for (int rr = 0; rr < G; ++rr)
+#pragma unroll
+                    for (int i = 0; i < VEC; ++i)
+                        if (r == rr) acc[rr * N + j * VEC + i] = g_combine<GOP>(acc[rr * N + j * VEC + i], m[i]);
+            }
+        }
+    };
+    // two positions per lane per step (independent gathers in flight)
+    for (int64_t k = b[0] + lane; k < b[G]; k += 64) {
+        add_edge(k);
+        if (k + 32 < b[G]) add_edge(k + 32);
+    }
+    seg_reduce_transposed<GOP, NT, 32>(acc, lane);
+    constexpr int SH = 5 - (NT >= 32 ? 5 : NT >= 16 ? 4 : NT >= 8 ? 3 : NT >= 4 ? 2 : NT >= 2 ? 1 : 0);
+    const int j = lane >> SH;                         // value index: row j / N, feature j % N
+    const int rr = j / N, col = j - rr * N;
+    if ((lane & ((1 << SH) - 1)) == 0 && col < op.W && v0 + rr < g.V) {
+        int64_t deg = 0;
+#pragma unroll
+        for (int r = 0; r < G; ++r)
+            if (r == rr) deg = b[r + 1] - b[r];
+        op.C[(v0 + rr) * op.c_ld + col] = g_finalize<GOP>(acc[0], deg);
+    }
+}
+
 cudaError_t launch_vertex_el(int kedge, int gather, const GraphArgs &g, const OpArgs &op, const LaunchCfg &c,
                              cudaStream_t s) {
     const int nc = (int)cdiv(op.W, c.vec);
+    const int ncp = nc <= 1 ? 1 : nc <= 2 ? 2 : nc <= 4 ? 4 : 8;     // NC instantiated
+    if (c.L == 32 && c.G > 1 && (c.G == 2 || c.G == 4 || c.G == 8) && c.G * ncp * c.vec <= 32) {
+        // segmented edge lanes: the warp's G rows share its lanes
+        const int64_t warps = cdiv(g.V, c.G);
+        const int64_t sgrid = cdiv(warps * 32, 256);
+#define UG_SEG(NCV, GV)                                                                                   \
+        UG_DISPATCH_KE(kedge, KE, UG_DISPATCH_RED(gather, GOP, {                                          \
+            if constexpr (GV * NCV * VEC <= 32) k_vertex_seg<KE, GOP, VEC, NCV, GV><<<(unsigned)sgrid, 256, 0, s>>>(g, op); \
+        }))
+#define UG_SEG_G(NCV)                                                                                     \
+        switch (c.G) {                                                                                    \
+        case 2: UG_SEG(NCV, 2); break;                                                                    \
+        case 4: UG_SEG(NCV, 4); break;                                                                    \
+        default: UG_SEG(NCV, 8); break;                                                                   \
+        }
+        UG_DISPATCH_VEC(c.vec, VEC, {
+            switch (ncp) {
+            case 1: UG_SEG_G(1); break;
+            case 2: UG_SEG_G(2); break;
+            case 4: UG_SEG_G(4); break;
+            default: UG_SEG_G(8); break;
+            }
+        });
+#undef UG_SEG_G
+#undef UG_SEG
+        return cudaGetLastError();
+    }
     const int64_t segs = cdiv(g.V, c.G);
     if (segs == 0) return cudaSuccess;
     const int64_t grid = cdiv(segs * c.L, 256);

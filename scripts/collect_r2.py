@@ -59,6 +59,14 @@ def main(tag):
     if os.path.exists(g(f"sweep_{tag}.jsonl")):
         shutil.copy(g(f"sweep_{tag}.jsonl"), os.path.join(R2, "sweep_r2_auto.jsonl"))
         run("scripts/fig12.py", os.path.join(R2, "sweep_r2_auto.jsonl"), out=os.path.join(R2, "fig12_auto_vs_best.md"))
+    # ncu --set full of the kernels changed in the second session (one launch each)
+    summ = {}
+    for name in ("C3_u_mul_e_sum", "C5_u_dot_v", "C2_copy_e_max"):
+        rep = g(f"prof_{name}_{tag}.ncu-rep")
+        if os.path.exists(rep):
+            summ[name] = json.loads(run("scripts/ncu_summary.py", "full", rep))
+    if summ:
+        json.dump(summ, open(os.path.join(R2, "ncu_kernels_r2b.json"), "w"), indent=1)
     for tool in ("memcheck", "racecheck", "synccheck"):
         src = g(f"sanitize_{tool}_{tag}.log")
         lines = [l for l in open(src).read().splitlines() if "=========" in l or "sanitize driver" in l]

@@ -23,7 +23,12 @@ SCHEDS = ["TV_G1_T1", "TV_G3_T4", "WV_G1_T1", "WV_G2_T2_F8", "TE_G1_T4", "TE_G5_
           "BV_G1", "BV_G3_B128", "BE_G64", "SV_G7", "SV_G64_F8", "SV_G5_F32", None]
 STAGED = ["SV_G7_M1", "SV_G7_A1", "SV_G16_F64_M1", "SV_G16_F32_A1"]       # aggregation ops only
 DOTT = ["SV_G7_F128", "SV_G16_F32"]                                          # u_dot_v ops only
-OPS = [("copy_lhs", "u", None, "sum", "v"), ("mul", "u", "e", "max", "v"), ("sub", "v", "u", "mean", "v"),
+# dst-sorted graph: the SV fast path (B addressing modes incl. the contiguous edge weight, FMA fold),
+# non-power-of-two column tiles, and the edge-lanes kernels (TV sub-warps, segmented WV)
+FAST = ["SV_G7", "SV_G64_F8", "SV_G16_F12"]
+FAST_EL = ["TV_G1_T8_E1", "TV_G1_T16_E1", "WV_G2_T1_E1", "WV_G4_T1_E1"]
+OPS = [("copy_lhs", "u", None, "sum", "v"), ("mul", "u", "e", "max", "v"), ("mul", "u", "e", "sum", "v"),
+       ("sub", "v", "u", "mean", "v"),
        ("div", "u", "e", "assign", "e"), ("dot", "u", "v", "sum", "v"), ("dot", "u", "v", "assign", "e")]
 
 
@@ -59,8 +64,10 @@ def main():
                     extra = DOTT
                 if eo != "dot" and c == "v" and F != 18:
                     extra = extra + ["WV_G1_T1_E1", "WV_G3_T1_E1"]      # edge-lanes (narrow F)
-                for s in SCHEDS + extra:
-                    gg = gs if s in STAGED else g
+                fast = []
+                if eo != "dot" and c == "v":
+                    fast = FAST + (FAST_EL if F != 18 else [])
+                for s, gg in [(s, gs if s in STAGED else g) for s in SCHEDS + extra] + [(s, gs) for s in fast]:
                     try:
                         ug.op_run(gg, eo, go, A=X, a_type=a, B=Bt, b_type=b, C=C, c_type=c, F=F, H=H, schedule=s)
                     except ug.UgError as err:

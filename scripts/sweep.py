@@ -53,7 +53,7 @@ def candidates(cls, F, E, quick=False):
         c += [f"TV_G{g}_T{t}" for g in (1, 4) for t in Ts]
         c += [f"WV_G{g}_T1" for g in (1, 2, 8)]
         if cls != "dot_agg" and F <= 32:
-            c += [f"WV_G{g}_T1_E1" for g in (1, 4)]       # lanes over in-edges (narrow F)
+            c += [f"WV_G{g}_T1_E1" for g in (1, 2, 4)]    # lanes over in-edges (narrow F); g > 1 segmented
             c += [f"TV_G1_T{t}_E1" for t in (8, 16)]       # 32 / t rows per warp, t edge lanes each
         c += [f"TE_G{g}_T{t}" for g in (1, 8, 32) for t in Ts if t >= 4]
         c += [f"WE_G{g}_T1" for g in (4, 32, 128)]

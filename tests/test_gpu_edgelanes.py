@@ -1,5 +1,6 @@
-"""GPU parity of the edge-lanes vertex schedules ("WV_Gg_T1_E1": a warp per row, "TV_Gg_Tt_E1": t in
-{8, 16} lanes per row, 32 / t rows per warp; k_vertex_el): every
+"""GPU parity of the edge-lanes vertex schedules ("WV_G1_T1_E1": a warp per row; "WV_Gg_T1_E1": g rows
+sharing a warp's lanes (k_vertex_seg); "TV_Gg_Tt_E1": t in {8, 16} lanes per row, 32 / t rows per
+warp; k_vertex_el): every
 aggregation op (all 32 message functions except dot x 4 reducers) in float mode (1e-5 * sum|terms|)
 and integer mode (bit-exact), widths 1..8 feature vectors, on an unsorted skewed multigraph
 (edge-id indirection, a hub row wider than the warp, zero in-degree rows)."""
@@ -29,10 +30,12 @@ def graph():
 @pytest.mark.parametrize("op", [o for o in all_ops() if o[4] == "v" and o[0] != "dot"], ids=name)
 def test_edgelanes_all_aggregations(graph, op, mode):
     V, E, src, dst, g = graph
-    for (F, H, ew) in ((20, 1, 1), (12, 3, 3), (32, 1, 32), (4, 1, 1)):
+    for (F, H, ew) in ((20, 1, 1), (12, 3, 3), (32, 1, 32), (4, 1, 1), (8, 1, 8)):
         A, B = operand_arrays(op, V, E, F, H, seed=F, mode=mode, edge_width=ew)
         ref, bound = run_oracle(op, V, src, dst, A, B, F, H)
-        for sch in ("WV_G1_T1_E1", "WV_G4_T1_E1", "TV_G1_T8_E1", "TV_G3_T16_E1"):
+        # WV_G{2,4,8}_T1_E1 with G * N <= 32 values: the segmented kernel (k_vertex_seg), else
+        # G rows one after another
+        for sch in ("WV_G1_T1_E1", "WV_G4_T1_E1", "WV_G2_T1_E1", "WV_G8_T1_E1", "TV_G1_T8_E1", "TV_G3_T16_E1"):
             got = run_gpu(ug, g, op, A, B, V, E, F, H, schedule=sch)
             assert_parity(op, got, ref, bound, mode == "int", what=f"{name(op)} {sch} F={F} H={H}")
 
