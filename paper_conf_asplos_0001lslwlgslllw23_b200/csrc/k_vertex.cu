@@ -131,8 +131,13 @@ __device__ __forceinline__ void seg_reduce_transposed(float (&v)[N], int lane) {
 // costs ceil(d / 2P) dependent gather steps instead of d / UF, which is what bounds small, skewed
 // graphs (C1 / C2) under the feature-lane schedules; P < 32 packs several light rows per warp
 // (fewer waves on graphs with more rows than resident warps, e.g. C2).
+// register budget: rows of <= 8 values in <= 2 vectors fit 6 CTAs / SM without spills (40 registers; C2's 19.7 K
+// rows at 16 lanes then take 1.4 waves instead of 2.1); wider rows stay uncapped (they spill)
+#ifndef UG_EL_MINB_NARROW
+#define UG_EL_MINB_NARROW 6
+#endif
 template <int KE, int GOP, int VEC, int NC, int P>
-__global__ void __launch_bounds__(256) k_vertex_el(GraphArgs g, OpArgs op, int G) {
+__global__ void __launch_bounds__(256, (NC * VEC <= 8 && NC <= 2 && (VEC >= 2 || KE == K_COPY)) ? UG_EL_MINB_NARROW : 1) k_vertex_el(GraphArgs g, OpArgs op, int G) {
     constexpr int N = NC * VEC;                       // values per lane (a power of two)
     constexpr int NOUT = N > P ? N / P : 1;           // totals a lane holds after the reduction
     const int64_t seg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / P;   // row group

@@ -62,13 +62,18 @@ def main(tag):
     # ncu --set full of the kernels changed in the second session (one launch each)
     summ = {}
     for name in ("C3_u_mul_e_sum", "C5_u_dot_v", "C2_copy_e_max"):
-        rep = g(f"prof_{name}_{tag}.ncu-rep")
-        if os.path.exists(rep):
-            summ[name] = json.loads(run("scripts/ncu_summary.py", "full", rep))
+        js = g(f"prof_{name}_{tag}.json")          # summarised on the box (scripts/gpu_evidence.sh)
+        if os.path.exists(js):
+            try:
+                summ[name] = json.load(open(js))
+            except ValueError:
+                pass
     if summ:
         json.dump(summ, open(os.path.join(R2, "ncu_kernels_r2b.json"), "w"), indent=1)
     for tool in ("memcheck", "racecheck", "synccheck"):
         src = g(f"sanitize_{tool}_{tag}.log")
+        if not os.path.exists(src):                # compute-sanitizer closed on the pool
+            continue
         lines = [l for l in open(src).read().splitlines() if "=========" in l or "sanitize driver" in l]
         open(os.path.join(P, "sanitizer", f"r2_{tool}.log"), "w").write("\n".join(lines[-3:]) + "\n")
     b = json.load(open(os.path.join(R2, "bench_line_r2.json")))
