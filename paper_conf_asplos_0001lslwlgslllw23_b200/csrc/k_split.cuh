@@ -38,8 +38,12 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
 #ifndef UG_BM6_UF
 #define UG_BM6_UF UG_BM2_UF
 #endif
+#ifndef UG_BM7_UF
+#define UG_BM7_UF UG_BM6_UF
+#endif
     constexpr int UF = BM == 0 || BM == 1 ? (VEC == 4 ? 8 : 16)
-                     : (BM >= 6 && KE != K_DIV) ? UG_BM6_UF
+                     : (BM == 7 && KE != K_DIV) ? UG_BM7_UF
+                     : (BM == 6 && KE != K_DIV) ? UG_BM6_UF
                      : (BM == 2 && KE != K_DIV) ? UG_BM2_UF : (VEC == 4 ? 4 : 8) / (KE == K_DIV ? 2 : 1);
     const float *__restrict__ Ab = op.A.p;          // warp-uniform base
     const uint64_t keep = l2_policy_evict_last();     // this tile's X column slab

@@ -131,10 +131,12 @@ __device__ __forceinline__ void seg_reduce_transposed(float (&v)[N], int lane) {
 // costs ceil(d / 2P) dependent gather steps instead of d / UF, which is what bounds small, skewed
 // graphs (C1 / C2) under the feature-lane schedules; P < 32 packs several light rows per warp
 // (fewer waves on graphs with more rows than resident warps, e.g. C2).
-// register budget: rows of <= 8 values in <= 2 vectors fit 6 CTAs / SM without spills (40 registers; C2's 19.7 K
-// rows at 16 lanes then take 1.4 waves instead of 2.1); wider rows stay uncapped (they spill)
+// register budget of narrow rows (<= 8 values in <= 2 vectors): capping them at 6 CTAs / SM (40
+// registers, spill-free; C2's 19.7 K rows at 16 lanes in 1.4 waves instead of 2.1) measured SLOWER
+// on every C1 / C2 case (C2 copy_e_max TV_G1_T16_E1 10.88 -> 11.54 us mean, u_mul_e_sum F = 8
+// 12.81 -> 14.41 us; profiles/r2/ab_el_r2fin2.jsonl): uncapped (1), kept as an A/B switch
 #ifndef UG_EL_MINB_NARROW
-#define UG_EL_MINB_NARROW 6
+#define UG_EL_MINB_NARROW 1
 #endif
 template <int KE, int GOP, int VEC, int NC, int P>
 __global__ void __launch_bounds__(256, (NC * VEC <= 8 && NC <= 2 && (VEC >= 2 || KE == K_COPY)) ? UG_EL_MINB_NARROW : 1) k_vertex_el(GraphArgs g, OpArgs op, int G) {
