@@ -680,6 +680,17 @@ def main():
                       "ncu_source": ncu_ent.get("source")}
         except (ValueError, OSError, KeyError, TypeError):
             traffic = None
+    # measured L2 -> SM read peak (scripts/probes/peaks.cu on this pool's B200s; the median of the
+    # probe's 96 MB runs): the direct denominator of the L2-bound kernel's achieved L2 -> SM bytes
+    pk = os.path.join(ROOT, "profiles", "r2", "peaks_r2.json")
+    if l2 and os.path.exists(pk):
+        try:
+            pkd = json.load(open(pk))
+            l2["l2_read_peak_gbs"] = pkd["l2_read_gbs_96MB"]
+            l2["frac_of_l2_read_peak"] = round(l2["achieved_gbs"] / pkd["l2_read_gbs_96MB"], 4)
+            l2["l2_peak_source"] = "profiles/r2/peaks_r2.json (" + pkd.get("how", "") + ")"
+        except (ValueError, OSError, KeyError, TypeError):
+            pass
 
     secondary = None
     headline_ops = None
