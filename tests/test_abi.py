@@ -170,7 +170,8 @@ def test_validate_rejects_width_mismatch():
 
 
 @pytest.mark.parametrize("text", ["TE_G1_T16", "WV_G4_T2", "TV_G1_T1", "WE_G64_T1", "BV_G2",
-                                  "BE_G256", "SV_G2048_F64", "SV_G1024_F128_B128_V4", "SV_G512_F64_P1"])
+                                  "BE_G256", "SV_G2048_F64", "SV_G1024_F128_B128_V4", "SV_G512_F64_P1",
+                                  "TV_G1_T16_E1", "WV_G4_T1_E1", "SV_G512_F120_P1", "SV_G4096_E1"])
 def test_schedule_text_roundtrip(text):
     s = ug.parse_schedule(text)
     assert ug.parse_schedule(ug.format_schedule(s)).strategy == s.strategy
@@ -321,3 +322,21 @@ def test_auto_schedule_always_resolves(cfg):
             A, B, C = _op_tensors(op, V, E, F, H)
             n = ug.launch_count(g, eo, gop, A=A, a_type=l, B=B, b_type=r, C=C, c_type=c, F=F, H=H)
             assert 1 <= n <= 4, (name(op), F, H, n)
+
+
+def test_round2_schedules_resolve_on_the_host():
+    """Round-2 schedule forms resolve (one launch each) or are rejected on the host: edge lanes
+    with P in {8, 16} lanes per row (TV) or a warp (WV, g rows segmented), and SV column tiles of
+    a non-power-of-two lane count (lanes past ftile / vec idle; at most 32)."""
+    src, dst = ugdata.graph("C1")
+    V, E = ugdata.CONFIGS["C1"].V, len(src)
+    g = host_graph(V, src, dst)
+    X, Y = torch.zeros(V, 16), torch.zeros(V, 16)
+    w = torch.zeros(E, 1)
+    kw = dict(A=X, a_type="u", C=Y, c_type="v")
+    for s in ("TV_G1_T8_E1", "TV_G2_T16_E1", "WV_G2_T1_E1", "WV_G4_T1_E1", "SV_G2_F12", "SV_G64_F24_P1"):
+        assert ug.launch_count(g, "copy_lhs", "sum", schedule=s, **kw) == 1, s
+        assert ug.launch_count(g, "mul", "sum", B=w, b_type="e", schedule=s, **kw) == 1, s
+    for bad in ("TV_G1_T4_E1", "TV_G1_T1_E1", "WV_G1_T2_E1", "SV_G2_F132"):
+        with pytest.raises(ug.UgError):
+            ug.launch_count(g, "copy_lhs", "sum", schedule=bad, **kw)
