@@ -27,9 +27,10 @@ namespace ug {
 // host checks rows * ld < 2^32).  The last, partial group of UF edges is predicated (its
 // missing slots re-read the row's last edge, an L1 hit, and are not combined), so short rows
 // never fall into a serial one-edge-at-a-time tail.  
-template <int KE, int GOP, int VEC, int BM>
+template <int KE, int GOP, int VEC, int BM, bool IDX = false>
 __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t k,
-                                                const int64_t k1, int f, int64_t cb, float (&acc)[VEC]) {
+                                                const int64_t k1, int f, int64_t cb, float (&acc)[VEC],
+                                                const int32_t *sidx = nullptr, int64_t kbase = 0) {
     // row gathers in flight per lane: 16 (measured +3 % over 8 on C5 at VEC 2), 8 for float4 rows;
     // half that when a B operand is loaded per edge (register budget of 40 for 6 CTAs / SM)
 #ifndef UG_BM2_UF
@@ -85,6 +86,10 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
                 s[q] = s_pf[q];
                 s_pf[q] = (uint32_t)ldg_i32_hint(g.col + min(k + UF + q, kl), stream);
             }
+        } else if constexpr (IDX) {
+            // column indices staged in this warp's shared-memory window (UG_SV_IDX_STAGE)
+#pragma unroll
+            for (int q = 0; q < UF; ++q) s[q] = (uint32_t)sidx[(PRED ? min(k + q, kl) : k + q) - kbase];
         } else {
 #pragma unroll
             for (int q = 0; q < UF; ++q) s[q] = (uint32_t)ldg_i32_hint(g.col + (PRED ? min(k + q, kl) : k + q), stream);
@@ -243,12 +248,68 @@ __device__ __forceinline__ void split_fast_assign(const GraphArgs &g, const OpAr
 #define UG_BM0_MINB 8
 #endif
 
+// Column-index staging (UG_SV_IDX_STAGE, the north star's "TMA or shared-memory staging of CSR
+// column-index tiles"; an A/B switch): when a whole warp serves one unit (L = 32), the unit's
+// col_idx[k0, k1) is copied into a per-warp shared-memory window of UG_IDX_WIN indices before the
+// gathers -- 1: by cp.async (LDGSTS, 4 bytes per lane), 2: by one 1-D bulk TMA copy
+// (cp.async.bulk ... mbarrier::complete_tx, issued by lane 0; the window starts at the aligned-down
+// 16-byte boundary, and the graph's col_idx allocation is padded so the rounded-up tail is in
+// bounds) -- and the in-edge loop reads its indices from shared memory.
+#ifndef UG_SV_IDX_STAGE
+#define UG_SV_IDX_STAGE 0
+#endif
+#define UG_IDX_WIN 512
+struct IdxStage {
+    int32_t *buf;        // this warp's window: UG_IDX_WIN + 4 indices, 16-byte aligned
+    uint32_t bar;        // its mbarrier (method 2)
+    uint32_t phase;
+};
+
+template <int KE, int GOP, int VEC, int BM>
+__device__ __forceinline__ void split_loop_staged(const GraphArgs &g, const OpArgs &op, int64_t v, int64_t k0,
+                                                  const int64_t k1, int f, int64_t cb, float (&acc)[VEC],
+                                                  IdxStage &st) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t kw = k0; kw < k1; kw += UG_IDX_WIN) {
+        const int64_t ke = min(k1, kw + (int64_t)UG_IDX_WIN);
+        int64_t kbase = kw;
+        if constexpr (UG_SV_IDX_STAGE == 1) {
+            const uint32_t dst = (uint32_t)__cvta_generic_to_shared(st.buf);
+            for (int64_t i = kw + lane; i < ke; i += 32)
+                asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst + (uint32_t)(i - kw) * 4u),
+                             "l"(g.col + i) : "memory");
+            asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+        } else {
+            const int64_t a0 = kw & ~(int64_t)3;           // 16-byte aligned start (col is 256-B aligned)
+            kbase = a0;
+            if (lane == 0) {
+                const uint32_t bytes = (uint32_t)(((ke - a0) * 4 + 15) & ~(int64_t)15);
+                const uint32_t dst = (uint32_t)__cvta_generic_to_shared(st.buf);
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(st.bar), "r"(bytes)
+                             : "memory");
+                asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                             ::"r"(dst), "l"(g.col + a0), "r"(bytes), "r"(st.bar) : "memory");
+            }
+            asm volatile(
+                "{\n\t.reg .pred p;\n\t"
+                "WAIT_%=:\n\t"
+                "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+                "@!p bra WAIT_%=;\n\t}" ::"r"(st.bar), "r"(st.phase) : "memory");
+            st.phase ^= 1u;
+        }
+        __syncwarp();
+        split_fast_loop<KE, GOP, VEC, BM, true>(g, op, v, kw, ke, f, cb, acc, st.buf, kbase);
+        __syncwarp();                                      // the window is refilled next
+    }
+}
+
 // One work unit (a chunk of <= G in-edges of one row, one VEC-wide column chunk per lane).
 // BM < 0: generic addressing (any operand types, eid); BM >= 0: the fast path with the B
 // operand's addressing mode fixed at compile time (see split_fast_loop).
 template <int KE, int GOP, int VEC, int BM>
 __device__ __forceinline__ void split_unit(const GraphArgs &g, const OpArgs &op, const int4 ch, const int f,
-                                           float *__restrict__ scratch, const int64_t sld) {
+                                           float *__restrict__ scratch, const int64_t sld, IdxStage *st = nullptr,
+                                           const bool store = true) {
     constexpr bool FAST = BM >= 0;
     constexpr int U = 4;                       // independent row gathers in flight per lane
     const int64_t v = ch.x;
@@ -276,7 +337,8 @@ __device__ __forceinline__ void split_unit(const GraphArgs &g, const OpArgs &op,
             // the row address is one IMAD + IMAD.WIDE from the (warp-uniform, L1-broadcast)
             // column index, so each in-edge costs ~6 instructions per lane.  The B operand's
             // addressing mode BM is a template parameter (a Dst_V operand is loaded once).
-            split_fast_loop<KE, GOP, VEC, BM>(g, op, v, k, k1, f, cb, acc);
+            if (UG_SV_IDX_STAGE && st) split_loop_staged<KE, GOP, VEC, BM>(g, op, v, k, k1, f, cb, acc, *st);
+            else split_fast_loop<KE, GOP, VEC, BM>(g, op, v, k, k1, f, cb, acc);
             k = k1;
         } else {
             for (; k + U <= k1; k += U) {
@@ -303,6 +365,7 @@ __device__ __forceinline__ void split_unit(const GraphArgs &g, const OpArgs &op,
         }
         // outputs are written once: evict_first keeps them from displacing the X slab in L2
         const uint64_t wpol = l2_policy_evict_first();
+        if (!store) return;
         if (ch.w < 0) {
             // sum needs no degree (an empty row's accumulator is already +0)
             const int64_t deg = GOP == UG_GATHER_SUM ? 1 : (int64_t)g.row_ptr[v + 1] - g.row_ptr[v];
@@ -399,6 +462,27 @@ __global__ void __launch_bounds__(256, (UG_ASSIGN_MINB > 0 && GOP == UG_GATHER_A
     const bool lane_ok = lane * VEC < ftile;       // false only for the idle lanes of a non-pow2 tile
     if constexpr (!MERGE) {
         // split rows (if any) are combined by k_split_fix, a second launch
+        if constexpr (UG_SV_IDX_STAGE != 0 && (BM == 0 || BM >= 6) && VEC == 4) {
+            if (L_log2 == 5) {                             // one unit per warp: stage its col_idx
+                __shared__ __align__(128) int32_t s_idx[8][UG_IDX_WIN + 4];
+                __shared__ __align__(8) uint64_t s_bar[8];
+                const int w = threadIdx.x >> 5;
+                IdxStage st{s_idx[w], (uint32_t)__cvta_generic_to_shared(&s_bar[w]), 0u};
+                if constexpr (UG_SV_IDX_STAGE == 2) {
+                    if ((threadIdx.x & 31) == 0) {
+                        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(st.bar) : "memory");
+                        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+                    }
+                    __syncwarp();
+                }
+                // every lane of the warp takes part in the staging; the idle lanes of a ragged last
+                // tile gather the tile's first columns (valid addresses) and store nothing
+                const bool act = f < op.W && lane_ok;
+                split_unit<KE, GOP, VEC, BM>(g, op, chunks[u - (int64_t)tile * n_chunks], act ? f : tile * ftile,
+                                             scratch, sld, &st, act);
+                return;
+            }
+        }
         if (f >= op.W || !lane_ok) return;
         split_unit<KE, GOP, VEC, BM>(g, op, chunks[u - (int64_t)tile * n_chunks], f, scratch, sld);
     } else {

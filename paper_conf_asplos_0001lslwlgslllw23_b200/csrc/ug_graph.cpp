@@ -56,7 +56,7 @@ ug_status finish_graph(ug_graph *g, const ug_allocator *alloc, cudaStream_t s) {
     if (cudaGetDevice(&g->device) != cudaSuccess) return set_error(UG_ERR_CUDA, "cudaGetDevice failed");
     const size_t rp = sizeof(int32_t) * (size_t)(V + 1), ne = sizeof(int32_t) * (size_t)g->E;
     g->d_row_ptr = (int32_t *)dev_alloc(g, rp, s);
-    g->d_col = (int32_t *)dev_alloc(g, ne, s);
+    g->d_col = (int32_t *)dev_alloc(g, ne + 64, s);   // +64 B: a 16-byte-rounded bulk copy of the tail stays in bounds
     g->d_dst = (int32_t *)dev_alloc(g, ne, s);
     if (!g->eid_identity) g->d_eid = (int32_t *)dev_alloc(g, ne, s);
     if (!g->d_row_ptr || !g->d_col || !g->d_dst || (!g->eid_identity && !g->d_eid))
