@@ -23,8 +23,15 @@ namespace ug {
 
 // O32: every row of P is addressable with a 32-bit element offset (V_src * ld < 2^32): a gather
 // address is one IMAD + IMAD.WIDE from the column index instead of 64-bit multiply / LEA pairs
+// message creation (u_dot_v, GOP assign) holds no running reduction: with 32-bit gather offsets its
+// widest instance fits 5 CTAs / SM spill-free (48 registers) -- C4 u_dot_v F = 128 69.6 -> 63.5 us,
+// F = 256 155.7 -> 139.2 us, C3 241.7 -> 225.3 us (profiles/r2/ab_r2t_dotsv_minb.jsonl); the
+// reductions keep UG_DOTSV_MINB (their NJ = 4 instance spills 144 B at 5)
+#ifndef UG_DOTSV_MINB_MSG
+#define UG_DOTSV_MINB_MSG 5
+#endif
 template <int GOP, int VEC, int NJ, bool O32>
-__global__ void __launch_bounds__(256, UG_DOTSV_MINB) k_dotsv(GraphArgs g, OpArgs op, bool a_is_src, const int4 *__restrict__ chunks,
+__global__ void __launch_bounds__(256, GOP == UG_GATHER_ASSIGN ? UG_DOTSV_MINB_MSG : UG_DOTSV_MINB) k_dotsv(GraphArgs g, OpArgs op, bool a_is_src, const int4 *__restrict__ chunks,
                                                   int64_t n_chunks, int L_log2, int w_log2,
                                                   float *__restrict__ scratch, int64_t sld) {
     constexpr int UE = NJ * VEC >= 16 ? 1 : 16 / (NJ * VEC);   // in-edges per step
