@@ -203,26 +203,42 @@ __device__ __forceinline__ void split_fast_assign(const GraphArgs &g, const OpAr
             for (int i = 0; i < VEC; ++i) m[i] = edge_fn<KE>(m[i], b[i]);
         }
     };
-    auto store = [&](int64_t kk, const float (&m)[VEC]) {
-        float *cp = op.C + kk * op.c_ld + f;
-        if (full_vec) st_vec_hint<VEC>(cp, m, stream);
-        else st_out<VEC>(cp, m, nout, op.c_vec);
+    // UG_ASSIGN_UNSWITCH: the loop unswitched on the (unit-invariant) store form, so full-vector
+    // stores carry no ragged-tail branches (36 -> 14 SASS instructions per edge) -- measured SLOWER
+    // (C4 u_add_v F = 128 157.7 -> 161.8 us, C3 F = 32 135.7 -> 143.3 us; profiles/r2/ab_r2u_assign.jsonl):
+    // message creation is bound by its write stream, not issue.  Off; kept as an A/B switch
+#ifndef UG_ASSIGN_UNSWITCH
+#define UG_ASSIGN_UNSWITCH 0
+#endif
+    auto run = [&](auto fv_tag) {
+        constexpr bool FV = decltype(fv_tag)::value;
+        auto store = [&](int64_t kk, const float (&m)[VEC]) {
+            float *cp = op.C + kk * op.c_ld + f;
+            if constexpr (FV) {
+                st_vec_hint<VEC>(cp, m, stream);
+            } else {
+                if (full_vec) st_vec_hint<VEC>(cp, m, stream);
+                else st_out<VEC>(cp, m, nout, op.c_vec);
+            }
+        };
+        for (; k + UF <= k1; k += UF) {
+            uint32_t sq[UF];
+#pragma unroll
+            for (int q = 0; q < UF; ++q) sq[q] = (uint32_t)ldg_i32_hint(g.col + k + q, stream);
+            float m[UF][VEC];
+#pragma unroll
+            for (int q = 0; q < UF; ++q) one(k + q, sq[q], m[q]);
+#pragma unroll
+            for (int q = 0; q < UF; ++q) store(k + q, m[q]);
+        }
+        for (; k < k1; ++k) {
+            float m[VEC];
+            one(k, (uint32_t)ldg_i32_hint(g.col + k, stream), m);
+            store(k, m);
+        }
     };
-    for (; k + UF <= k1; k += UF) {
-        uint32_t sq[UF];
-#pragma unroll
-        for (int q = 0; q < UF; ++q) sq[q] = (uint32_t)ldg_i32_hint(g.col + k + q, stream);
-        float m[UF][VEC];
-#pragma unroll
-        for (int q = 0; q < UF; ++q) one(k + q, sq[q], m[q]);
-#pragma unroll
-        for (int q = 0; q < UF; ++q) store(k + q, m[q]);
-    }
-    for (; k < k1; ++k) {
-        float m[VEC];
-        one(k, (uint32_t)ldg_i32_hint(g.col + k, stream), m);
-        store(k, m);
-    }
+    if (UG_ASSIGN_UNSWITCH && full_vec) run(std::true_type{});
+    else run(std::false_type{});
 }
 
 // BM = 2 (per-edge scalar B, e.g. u_mul_e_sum): 6 CTAs / SM (40 registers, spill-free) for sum /
