@@ -211,8 +211,12 @@ __global__ void __launch_bounds__(256, UG_DAW_MINB) k_dotattn(GraphArgs g, DotAt
 #define UG_DAH_MINB 4   // resident CTAs per SM the register budget is sized for
 #endif
 
+// float / float2 slices fit 5 CTAs / SM spill-free (48 registers); float4 slices spill there
+#ifndef UG_DAH_MINB_NARROW
+#define UG_DAH_MINB_NARROW UG_DAH_MINB
+#endif
 template <int VEC, int UE>
-__global__ void __launch_bounds__(256, UG_DAH_MINB) k_dotattn_heads(GraphArgs g, DotAttnArgs a, const int4 *__restrict__ chunks,
+__global__ void __launch_bounds__(256, VEC <= 2 ? UG_DAH_MINB_NARROW : UG_DAH_MINB) k_dotattn_heads(GraphArgs g, DotAttnArgs a, const int4 *__restrict__ chunks,
                                                        int n_chunks, int n_units, int L_log2, int w_log2,
                                                        float *__restrict__ scratch, int64_t sld) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
