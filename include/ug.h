@@ -112,9 +112,13 @@ typedef struct {
     int32_t group;          /* G: units per thread/warp group (V/E grouping);
                                UG_SV: max edges per row chunk                                    */
     int32_t tile;           /* T: feature tiling: threads (TV/TE) or warps (WV/WE)
-                               sharing one unit's features                                       */
+                               sharing one unit's features; with UG_SCHED_EDGELANES the lanes that
+                               share one row's in-edges (TV: 8 or 16; WV: 1 warp)                */
     int32_t block_threads;  /* CTA size (0 -> 256)                                              */
-    int32_t ftile;          /* column-tile width for L2 blocking, tile-major grid order; 0 = off */
+    int32_t ftile;          /* column-tile width for L2 blocking, tile-major grid order; 0 = off.
+                               UG_SV: a multiple of vec with ftile / vec <= 32 lanes (rounded up
+                               to a power of two, the extra lanes idle); UG_SV dot between a Src_V
+                               and a Dst_V operand: 32 / 64 / 128 selects the column-tiled kernel */
     int32_t vec;            /* feature vector width 1/2/4; 0 -> widest the layout allows        */
     int32_t flags;          /* UG_SCHED_PACK | UG_SCHED_TMA | UG_SCHED_ASYNC | UG_SCHED_EDGELANES.  UG_SCHED_PACK (SV only): first stage a full-width Src_V operand whose
                                rows are not 128-byte aligned into an aligned scratch copy, so each
