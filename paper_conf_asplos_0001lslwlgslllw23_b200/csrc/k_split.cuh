@@ -156,8 +156,19 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
         }
     };
     for (; k + UF <= k1; k += UF) group(std::false_type{}, std::integral_constant<int, UF>{});
-    // the last, partial group: predicated half-groups (fewer registers), not a serial tail
+    // the last, partial group: predicated half-groups (fewer registers), not a serial tail.
+    // UG_SV_TAIL_FULL: a remainder of more than UF / 2 edges takes ONE predicated full-size group
+    // (one dependent round trip instead of two for short rows; A/B switch)
     constexpr int UH = UF / 2 > 0 ? UF / 2 : 1;
+#ifndef UG_SV_TAIL_FULL
+#define UG_SV_TAIL_FULL 0
+#endif
+    if constexpr (UG_SV_TAIL_FULL && UF > 1) {
+        if (k1 - k > UH) {
+            group(std::true_type{}, std::integral_constant<int, UF>{});
+            k = k1;
+        }
+    }
     for (; k < k1; k += UH) group(std::true_type{}, std::integral_constant<int, UH>{});
 }
 
