@@ -103,7 +103,7 @@ __device__ __forceinline__ void split_fast_loop(const GraphArgs &g, const OpArgs
         // UG_MUL_FMA: a per-edge scalar weight folded into the sum by FMA (the message x * w is then
         // rounded together with the add, not on its own -- inside R11's 1e-5 * sum|terms| bound,
         // exact in integer mode).  On with the contiguous-weight loops: C5 u_mul_e_sum 19.19 ->
-        // 18.71 ms, C3 F = 128 256.3 -> 254.2 us (profiles/r2/ab_r2l.jsonl; r2 with BM 2 it lost)
+        // 18.71 ms, C3 F = 128 256.3 -> 254.2 us (profiles/r2/ab_s2_r2l.jsonl; r2 with BM 2 it lost)
         constexpr bool FMA_W = UG_MUL_FMA && BM >= 6 && KE == K_MUL && (GOP == UG_GATHER_SUM || GOP == UG_GATHER_MEAN);
         if constexpr (FMA_W) {
             float wq[UF];
@@ -267,7 +267,7 @@ __device__ __forceinline__ void split_fast_assign(const GraphArgs &g, const OpAr
 #endif
 // BM = 7: the BM 6 loop at 8 CTAs / SM (32 registers) for sum / mean on short-chunk graphs with
 // many waves -- C3 u_mul_e_sum F = 128 268.5 -> 252.2 us, C4 92.4 -> 86.3 us, but C5 (long chunks)
-// 19.5 -> 21.3 ms and C2 (one wave) 13.6 -> 15.6 us (profiles/r2/ab_r2i.jsonl); chosen at launch
+// 19.5 -> 21.3 ms and C2 (one wave) 13.6 -> 15.6 us (profiles/r2/ab_s2_r2i.jsonl); chosen at launch
 #ifndef UG_BM7_MINB
 #define UG_BM7_MINB 8
 #endif
