@@ -66,7 +66,9 @@ struct SoftState {
 // One pass over a chunk's edges k0 .. k1 (contiguous CSR positions): U row gathers in flight
 // per lane, the next group's column indices prefetched while the current group computes, and
 // the running max updated once per group of U edges (one rescale per group).
-template <int VEC, int U>
+// O32: el and z rows addressable with 32-bit element offsets (V_src * ld < 2^32, checked on the
+// host): one IMAD + IMAD.WIDE per gather instead of a 64-bit multiply and LEA pair
+template <int VEC, int U, bool O32 = false>
 __device__ __forceinline__ void gat_walk(const GraphArgs &g, const GatArgs &a, int k0, int k1, int h, int f,
                                          bool active, float erv, SoftState<VEC> &st) {
     // padding slots read row 0 (cache-hot) and are masked by t = -inf: no branches
@@ -101,8 +103,13 @@ __device__ __forceinline__ void gat_walk(const GraphArgs &g, const GatArgs &a, i
             t[q] = tt[0];
             ldg_vec_hint<VEC>(zb + (int64_t)u * a.ld_z, zr[q], keep);
 #else
-            t[q] = __ldg(eb + (int64_t)u * a.ld_el);
-            ldg_vec<VEC>(zb + (int64_t)u * a.ld_z, zr[q]);
+            if constexpr (O32) {
+                t[q] = __ldg(a.el + (u * (uint32_t)a.ld_el + (uint32_t)h));
+                ldg_vec<VEC>(a.z + (u * (uint32_t)a.ld_z + (uint32_t)(active ? f : 0)), zr[q]);
+            } else {
+                t[q] = __ldg(eb + (int64_t)u * a.ld_el);
+                ldg_vec<VEC>(zb + (int64_t)u * a.ld_z, zr[q]);
+            }
 #endif
         }
 #undef UG_GAT_COL
@@ -165,7 +172,7 @@ __device__ __forceinline__ void gat_store(const GatArgs &a, int64_t v, int f, co
 // MB = resident CTAs per SM the register budget is sized for: 6 (40 registers) for float4 slices of
 // large graphs, 1 (no cap, 48) otherwise -- r2al: C4 H = 8 F = 128 148.8 -> 128.3 us, C3 H = 4
 // F = 64 224 -> 190 us, but C2 14.7 -> 15.7 us, hence by grid size
-template <int VEC, int U, bool ATTN, int MB>
+template <int VEC, int U, bool ATTN, int MB, bool O32>
 __global__ void __launch_bounds__(256, MB) k_gat(GraphArgs g, GatArgs a, int L_log2, int n_tiles,
                                              const int4 *__restrict__ chunks, int64_t n_chunks,
                                              const int4 *__restrict__ split, const int32_t *__restrict__ slot_row,
@@ -189,7 +196,7 @@ __global__ void __launch_bounds__(256, MB) k_gat(GraphArgs g, GatArgs a, int L_l
     const float erv = __ldg(a.er + v * a.ld_er + h);
     SoftState<VEC> st;
     st.init();
-    gat_walk<VEC, U>(g, a, ch.y, ch.z, h, f, active, erv, st);
+    gat_walk<VEC, U, O32>(g, a, ch.y, ch.z, h, f, active, erv, st);
     if (ch.w < 0) {                                   // the row is one chunk: finalise here
         if (active) gat_store<VEC>(a, v, f, st, ch.z == ch.y);
         if constexpr (ATTN) {
@@ -234,6 +241,9 @@ __global__ void __launch_bounds__(256, MB) k_gat(GraphArgs g, GatArgs a, int L_l
     }
 }
 
+#ifndef UG_GAT_O32
+#define UG_GAT_O32 1
+#endif
 cudaError_t launch_gat(const GraphArgs &g, const GatArgs &a, int vec, int L, const SplitPlan &plan,
                        const int32_t *slot_row, float *sacc, float *sst, int64_t sld, int64_t nfc,
                        int32_t *counters, cudaStream_t s) {
@@ -246,11 +256,24 @@ cudaError_t launch_gat(const GraphArgs &g, const GatArgs &a, int vec, int L, con
     const int4 *chunks = reinterpret_cast<const int4 *>(plan.d_chunk);
     const int4 *split = reinterpret_cast<const int4 *>(plan.d_split);
     const bool big = grid >= 4096;
+    const bool o32 = UG_GAT_O32 && (uint64_t)g.V_src * (uint64_t)a.ld_z < (1ull << 32) &&
+                     (uint64_t)g.V_src * (uint64_t)a.ld_el < (1ull << 32);
 #define UG_GAT_LAUNCH(ATTN_, MB_)                                                                               \
-    k_gat<VEC, (VEC == 4 ? 4 : 8), ATTN_, MB_><<<(unsigned)grid, block, 0, s>>>(                               \
-        g, a, L_log2, n_tiles, chunks, plan.n_chunks, split, slot_row, sacc, sst, sld, nfc, counters)
+    do {                                                                                                        \
+        if (o32)                                                                                                \
+            k_gat<VEC, (VEC == 4 ? 4 : 8), ATTN_, MB_, true><<<(unsigned)grid, block, 0, s>>>(                 \
+                g, a, L_log2, n_tiles, chunks, plan.n_chunks, split, slot_row, sacc, sst, sld, nfc, counters);  \
+        else                                                                                                    \
+            k_gat<VEC, (VEC == 4 ? 4 : 8), ATTN_, MB_, false><<<(unsigned)grid, block, 0, s>>>(                \
+                g, a, L_log2, n_tiles, chunks, plan.n_chunks, split, slot_row, sacc, sst, sld, nfc, counters);  \
+    } while (0)
+    // 32-bit offsets only in the uncapped instance: at 6 CTAs / SM they spill 56 B and lose 6-12 %
+    // (C4 H = 8 F = 128 127.3 -> 137.4 us), uncapped they win (C2 H = 8 14.67 -> 13.66 us;
+    // profiles/r2/ab_r2gat.jsonl)
+    const bool o32_small = o32;
     UG_DISPATCH_VEC(vec, VEC, {
         if constexpr (VEC == 4) {
+            const bool o32 = o32_small && !big;
             if (a.attn) { if (big) UG_GAT_LAUNCH(true, 6); else UG_GAT_LAUNCH(true, 1); }
             else { if (big) UG_GAT_LAUNCH(false, 6); else UG_GAT_LAUNCH(false, 1); }
         } else {
